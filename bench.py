@@ -1,0 +1,349 @@
+"""Benchmark of the mSTAMP hot path (BASELINE.json metric: d*n^2 matrix-profile cells*dims/s).
+
+A "step" = one whole pass of the hot path (precompute -> fused diagonal kernel ->
+finalize) over the workload, inputs resident in HBM.  Default workload: BASELINE
+config C2 (self-join, d=16, n=65536, m=128, seeded random walk + planted motif), the
+configuration the metric is quoted on, FP32 headline; every precision is also timed
+and reported under "per_precision".
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--precision fp32] [--config C2]
+  python bench.py --impl reference ...   (the FP64 CPU oracle on host cores, sampled rows)
+
+Multi-GPU (torchrun, one process per GPU): each rank computes its equal-cell diagonal
+band, one NCCL MINLOC all-reduce merges the partial profiles (the path's only exchange);
+time = max over ranks, value = total d*n^2 / time ("scaling": "strong": the job is
+fixed, bands shrink with N).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_ipps_juryl022_b200 import datagen  # noqa: E402
+
+PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
+METRIC = "matrix-profile cells*dims/sec (d*n^2/s)"
+UNIT = "cells*dims/s"
+SM_COUNT = 148
+ALU_LANES = 64          # ALU-pipe lanes per SM per clock (FMNMX/FSETP/FSEL), B300_MICROARCH "alu rt=2/SMSP"
+NOMINAL_SM_MHZ = 1965.0
+
+
+def batcher_ce(N: int) -> int:
+    """Comparators of Batcher's odd-even merge sort network on N inputs (as sort_net builds it)."""
+    c = 0
+    p = 1
+    while p < N:
+        k = p
+        while k >= 1:
+            j = k % p
+            while j + k < N:
+                for i in range(k):
+                    if i + j + k < N and (i + j) // (2 * p) == (i + j + k) // (2 * p):
+                        c += 1
+                j += 2 * k
+            k >>= 1
+        p <<= 1
+    return c
+
+
+def alu_ops_per_cell_dim(d: int, self_join: bool) -> float:
+    """Algorithmic ALU-pipe ops per computed cell*dim: the d-way sort
+    network (2 FMNMX per comparator, padded to a power of two) + 1 threshold compare per
+    profile side updated (row; + column for the self-join)."""
+    dp = 1
+    while dp < d:
+        dp <<= 1
+    return 2.0 * batcher_ce(dp) / d + (2.0 if self_join else 1.0)
+
+
+def computed_cells(n: int, e: int, self_join: bool) -> int:
+    if self_join:
+        k = n - e - 1
+        return k * (k + 1) // 2 if k > 0 else 0
+    return n * n
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+        self.t = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                sm.append(float(f[1]))
+                smax.append(float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def load_peaks():
+    try:
+        with open(PEAKS_PATH) as f:
+            return json.load(f), "measured"
+    except OSError:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "sm_max_mhz": NOMINAL_SM_MHZ}, "fallback"
+
+
+def launches_per_step(prec: str, self_join: bool) -> int:
+    # check_finite (1 per series) + precompute (pre_stats, pre_diff [+ to_f32]) per series
+    # + init_keys + mp_diag + [keys64_to_ext] + finalize
+    series = 1 if self_join else 2
+    pre = 2 if prec == "fp64" else 3
+    return series * (1 + pre) + 1 + 1 + (1 if prec == "fp64" else 0) + 1
+
+
+# ---------------------------------------------------------------------------- CPU oracle leg
+def oracle_sample(cfg, target_s: float = 15.0, max_rows: int = 4096):
+    """Time the FP64 oracle (as it stands) on sampled query rows of the workload.
+    Returns (cell*dims per second, rows, seconds, threads)."""
+    import oracle
+    oracle.build()
+    T, Tr, m, e, n, d = cfg["T"], cfg["Tr"], cfg["m"], cfg["exclusion"], cfg["n"], cfg["d"]
+    threads = os.cpu_count() or 1
+    rng = np.random.default_rng(0)
+    rows = np.sort(rng.choice(n, size=min(threads, n), replace=False))
+    t0 = time.perf_counter()
+    oracle.mstamp(T, m, e, Tr=Tr, rows=rows, nthreads=threads)
+    dt = time.perf_counter() - t0
+    nr = int(min(max_rows, max(len(rows), len(rows) * target_s / max(dt, 1e-6))))
+    nr = max(threads, (nr // threads) * threads)
+    rows = np.sort(rng.choice(n, size=min(nr, n), replace=False))
+    t0 = time.perf_counter()
+    oracle.mstamp(T, m, e, Tr=Tr, rows=rows, nthreads=threads)
+    dt = time.perf_counter() - t0
+    cells = len(rows) * n * d          # each sampled row: all n reference windows x d dims
+    return cells / dt, len(rows), dt, threads
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    cfg = datagen.make(args.config)
+    vals = []
+    for _ in range(args.warmup):
+        oracle_sample(cfg, target_s=2.0)
+    meta = None
+    for _ in range(args.steps):
+        v, nr, dt, th = oracle_sample(cfg, target_s=args.ref_seconds)
+        vals.append(v)
+        meta = (nr, dt, th)
+    value = statistics.mean(vals)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": meta[1] * 1e3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": config_json(args, cfg),
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": meta[2], "kind": "oracle",
+                             "sample": f"{meta[0]} random query rows x all n reference windows per step"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def config_json(args, cfg):
+    return {"workload": f"{args.config}: {'self' if cfg['Tr'] is None else 'AB'}-join d={cfg['d']} "
+                        f"n={cfg['n']} m={cfg['m']} exclusion={cfg['exclusion']}",
+            "d": cfg["d"], "n": cfg["n"], "m": cfg["m"], "exclusion": cfg["exclusion"],
+            "join": "self" if cfg["Tr"] is None else "ab", "precision": args.precision,
+            "parallelism": f"diagonal-bands x{args.gpus}",
+            "l2": "flushed between timed steps (256 MiB write)"}
+
+
+# ---------------------------------------------------------------------------- GPU leg
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--precision", default="fp32")
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--impl", default="native", choices=["native", "reference"])
+    ap.add_argument("--ref-seconds", type=float, default=15.0)
+    ap.add_argument("--no-per-precision", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_juryl022_b200 import mstamp
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    cfg = datagen.make(args.config)
+    d, n, m, e = cfg["d"], cfg["n"], cfg["m"], cfg["exclusion"]
+    self_join = cfg["Tr"] is None
+    T = torch.from_numpy(cfg["T"]).to(dev)
+    Tr = None if self_join else torch.from_numpy(cfg["Tr"]).to(dev)
+    ctx = mstamp.Context(local)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream(dev)
+
+    def one_step(prec):
+        """One pass of the whole hot path; returns (device ms, main-kernel ms)."""
+        P = torch.empty(d, n, dtype=torch.float64, device=dev)
+        I = torch.empty(d, n, dtype=torch.int64, device=dev)
+        flush.fill_(1)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        if world == 1:
+            ctx.compute_device(T, m, P, I, prec, e, Tr=Tr, stream=stream)
+        else:
+            keys = torch.empty(mstamp.key_words(d, n, prec), dtype=torch.int64, device=dev)
+            ctx.partial_device(T, m, keys, rank, world, prec, e, Tr=Tr, stream=stream)
+            mstamp.merge_partials(ctx, keys, d, n, prec)
+            if rank == 0:
+                ctx.finalize_device(d, n, keys, P, I, prec, stream=stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        kms, _ = ctx.last_timing()
+        return e0.elapsed_time(e1), kms
+
+    def timed(prec, steps, warm, sample_clocks=False):
+        for _ in range(warm):
+            one_step(prec)
+        cs = ClockSampler(local) if sample_clocks else None
+        if cs:
+            cs.start()
+            time.sleep(0.3)
+        ms, kms = [], []
+        for _ in range(steps):
+            a, b = one_step(prec)
+            ms.append(a)
+            kms.append(b)
+        clocks = cs.stop() if cs else None
+        tot = torch.tensor([sum(ms)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+        return tot.item() / steps, statistics.mean(kms), clocks
+
+    ms, kms, clocks = timed(args.precision, args.steps, args.warmup, sample_clocks=True)
+    dn2 = d * n * n
+    value = dn2 / (ms * 1e-3)
+
+    per_prec = {}
+    if not args.no_per_precision:
+        for prec in ("fp64", "fp32"):
+            if prec == args.precision:
+                per_prec[prec] = {"value": value, "ms_per_step": ms, "main_kernel_ms": kms}
+                continue
+            p_ms, p_kms, _ = timed(prec, max(1, min(args.steps, 3)), 1)
+            per_prec[prec] = {"value": dn2 / (p_ms * 1e-3), "ms_per_step": p_ms, "main_kernel_ms": p_kms}
+
+    # e2e through the C-ABI host entry point (pinned host buffers, H2D + D2H inside)
+    e2e = None
+    if world == 1:
+        Th = torch.from_numpy(cfg["T"]).pin_memory().numpy()
+        Trh = None if self_join else torch.from_numpy(cfg["Tr"]).pin_memory().numpy()
+        ctx.compute(Th, m, args.precision, e, Tr=Trh)
+        ts = []
+        for _ in range(args.steps):
+            flush.fill_(1)
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            ctx.compute(Th, m, args.precision, e, Tr=Trh)
+            ts.append(time.perf_counter() - t0)
+        L = n + m - 1
+        e2e = {"value": dn2 / statistics.mean(ts), "unit": UNIT,
+               "h2d_bytes_per_step": d * L * 8 * (1 if self_join else 2), "d2h_bytes_per_step": 2 * d * n * 8,
+               "ms_per_step": statistics.mean(ts) * 1e3}
+
+    if rank == 0:
+        peaks, src = load_peaks()
+        cells = computed_cells(n, e, self_join)
+        if world > 1:
+            cells = cells  # each rank's kernel time is for its band; report job-level ops / max time
+        ops = alu_ops_per_cell_dim(d, self_join) * cells * d
+        peak_tops = SM_COUNT * ALU_LANES * NOMINAL_SM_MHZ * 1e6 / 1e12
+        achieved = ops / (kms * 1e-3) / 1e12 if kms > 0 else None
+        roof = {"bound": "alu", "achieved": achieved, "peak": peak_tops, "unit": "Tops/s",
+                "frac": achieved / peak_tops if achieved else None, "traffic": None,
+                "kernel": "mp_diag", "ops_per_cell_dim": alu_ops_per_cell_dim(d, self_join),
+                "computed_cell_dims": cells * d,
+                "peak_basis": f"148 SM x 64 ALU lanes/clk x {NOMINAL_SM_MHZ:.0f} MHz (derived; MEASURED_PEAKS {src} "
+                              "has no ALU figure)"}
+        cpu = None
+        if not args.no_cpu_baseline and world == 1:
+            v, nr, dt, th = oracle_sample(cfg, target_s=args.ref_seconds)
+            cpu = {"value": v, "unit": UNIT, "cores": th, "kind": "oracle",
+                   "sample": f"{nr} random query rows x all {n} reference windows ({dt:.1f} s)"}
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+                "vs_baseline": None, "dtype": {"fp64": "f64", "fp32": "f32"}.get(args.precision, args.precision),
+                "data": "synthetic", "config": config_json(args, cfg), "roofline": roof, "cpu_baseline": cpu,
+                "e2e": e2e, "gpu_launches": launches_per_step(args.precision, self_join) * args.steps,
+                "clocks": clocks, "per_precision": per_prec,
+                "computed_cells_per_s": cells * d / (ms * 1e-3)}
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,138 @@
+/*
+ * include/mp.h -- C ABI of the B200-native mSTAMP hot path (libmstamp_b200.so).
+ *
+ * What it computes (PAPER.md = /root/reference/PAPER.md, Ju et al., IPDPS 2022):
+ *   For query series Tq and reference series Tr (both d x L, L = n + m - 1,
+ *   PAPER.md:L461-473, footnote L515-516: n = number of subsequences), for every
+ *   cell (i, j) of the n x n subsequence grid and every dimension k:
+ *     QT  by the streaming recurrence along each diagonal        Eq. (1)
+ *     D   = sqrt(2 m (1 - QT d_q^-1 d_r^-1))                     Eq. (1)
+ *     D'  = sort(D[i,j,:]) ascending;  D'' = inclusive mean      Eq. (2)
+ *     P[k][i] = min_j D''[i,j,k],  I[k][i] = argmin_j            Eq. (3)
+ *   Self-join (Tr == NULL): cells with |i - j| <= exclusion are skipped
+ *   (reading G1); AB-join: every j, query profile only.
+ *   Ties: the lowest j wins (G2).  Rows with no admissible j: P = +inf, I = -1 (G3).
+ *
+ * Layouts: every matrix is row-major "d rows x n (or L) columns", i.e. element
+ *   (k, i) at [k * n + i]; dimension k contiguous (the paper's "dimension-wise
+ *   layout", L662-666).
+ * Precision modes (Fig. 1 table, Sec. III-C): see mp_precision.
+ * Ownership: the caller owns T, Tr, P, I (host memory for mp_compute, device memory
+ *   for the _device variants); the context owns all device scratch and the
+ *   per-device streams it creates, caches scratch by shape, frees it in mp_free.
+ * Errors: every call returns mp_status; nothing aborts or throws across the ABI.
+ *   On a non-OK status outputs are unspecified and no memory is leaked;
+ *   mp_last_error(ctx) returns a message.
+ * Threading: one context per host thread.
+ * Determinism: for a given (inputs, prec, reseed interval) the outputs are
+ *   bit-identical for any number of GPUs / ranks and any launch order (fixed
+ *   tiling; lexicographic (value, index) minimum is order-independent).
+ */
+#ifndef MP_H_
+#define MP_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    MP_OK = 0,
+    MP_ERR_INVALID = 1,     /* bad argument: NULL, d<1, n<2, m<2, non-finite input, n >= 2^31, d > MP_MAX_D */
+    MP_ERR_NOMEM = 2,       /* device or host allocation failed */
+    MP_ERR_CUDA = 3,        /* CUDA runtime error (message in mp_last_error) */
+    MP_ERR_NCCL = 4,        /* reserved: collectives run in the caller's process group */
+    MP_ERR_UNSUPPORTED = 5  /* valid request this build does not implement (e.g. precision x d) */
+} mp_status;
+
+typedef enum {
+    MP_FP64 = 0,   /* precalculation FP64, main loop FP64           (L426-428, L764-766) */
+    MP_FP32 = 1,   /* precalculation FP32, main loop FP32           (L430-432, L771-772) */
+    MP_FP16 = 2,   /* precalculation FP16, main loop FP16           (L434-436, L773-776) */
+    MP_MIXED = 3   /* precalculation FP32, main loop FP16           (L438-440, L777-785) */
+} mp_precision;
+
+#define MP_MAX_D 1024
+
+typedef struct mp_ctx mp_ctx;   /* opaque */
+
+typedef struct {
+    int device;             /* CUDA device ordinal this context drives (one process per GPU) */
+    int64_t reseed_h[4];    /* re-seed interval H (rows) per mp_precision; 0 -> default */
+} mp_config;
+
+/* Create a context on cfg->device (cfg == NULL -> device 0, defaults). */
+mp_status mp_init(mp_ctx** out, const mp_config* cfg);
+
+/* Free all device memory and streams owned by ctx.  NULL-safe. */
+void mp_free(mp_ctx* ctx);
+
+/* Message for the last non-OK status on ctx (static string if ctx == NULL). */
+const char* mp_last_error(const mp_ctx* ctx);
+
+/* Library version string. */
+const char* mp_version(void);
+
+/*
+ * Whole matrix profile on the context's device, HOST buffers.
+ *   T   [d x L] query series (FP64, L = n + m - 1); Tr: reference series, same
+ *       shape, or NULL for a self-join.
+ *   exclusion: self-join skips |i - j| <= exclusion; < 0 -> ceil(m / 4); ignored for AB.
+ *   P   [d x n] out: P[k*n + i] = mean of the k+1 smallest per-dimension distances
+ *       of query window i to its nearest reference window.
+ *   I   [d x n] out: that reference window's index j, or -1 if none.
+ * Includes the host->device copy of T (and Tr) and the device->host copy of P, I.
+ */
+mp_status mp_compute(mp_ctx* ctx, const double* T, const double* Tr,
+                     int64_t d, int64_t n, int64_t m, mp_precision prec,
+                     int64_t exclusion, double* P, int64_t* I);
+
+/* Same as mp_compute with DEVICE pointers on the caller's CUDA stream (may be NULL). */
+mp_status mp_compute_device(mp_ctx* ctx, void* cuda_stream, const double* dT, const double* dTr,
+                            int64_t d, int64_t n, int64_t m, mp_precision prec,
+                            int64_t exclusion, double* dP, int64_t* dI);
+
+/*
+ * Multi-GPU building blocks (one process per GPU; the caller's process group does
+ * the collective -- the only exchange step of the path, Pseudocode 2 l.6-8,
+ * PAPER.md:L738-740, replaced by an on-device MINLOC all-reduce).
+ *
+ * mp_partial_device: compute the band `rank` of `world` equal-cell diagonal
+ *   bands and leave the partial profile as merge keys in dKeys.
+ *   dKeys must hold mp_key_words(d, n, prec) int64 words on the device.
+ *   Key format (bit-exact lexicographic (value, index) order):
+ *     FP32/FP16/MIXED: one int64 per (k, i) = (float bits of the k-dim distance SUM << 32) | j;
+ *                      reduce with MIN over int64.
+ *     FP64: two int64 planes; plane 0 = double bits of the distance SUM (reduce MIN),
+ *           plane 1 = index; call mp_key_mask_device between the two MIN reductions.
+ *   Empty entries are INT64_MAX.
+ */
+int64_t   mp_key_words(int64_t d, int64_t n, mp_precision prec);
+mp_status mp_partial_device(mp_ctx* ctx, void* cuda_stream, const double* dT, const double* dTr,
+                            int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
+                            int rank, int world, int64_t* dKeys);
+/* FP64 merge step 2: where plane0 != global plane0 (dGlobalV), set the index to INT64_MAX. */
+mp_status mp_key_mask_device(mp_ctx* ctx, void* cuda_stream, int64_t d, int64_t n,
+                             int64_t* dKeys, const int64_t* dGlobalV);
+/* Merged keys -> P (double, divided by k+1) and I (int64, -1 for empty). */
+mp_status mp_finalize_device(mp_ctx* ctx, void* cuda_stream, int64_t d, int64_t n, mp_precision prec,
+                             const int64_t* dKeys, double* dP, int64_t* dI);
+
+/*
+ * Host-side scheduler query (no GPU needed): the first diagonal-block index of
+ * band `rank` of `world` and the number of cells per band (cells = (i,j) pairs
+ * the band computes).  Bands are contiguous diagonal ranges with equal cell
+ * counts up to one block.  block_begin/cells arrays have world+1 / world entries.
+ */
+mp_status mp_plan_bands(int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
+                        int self_join, int world, int64_t* block_begin, int64_t* cells);
+
+/* Kernel timing of the last mp_compute* / mp_partial_device call on ctx (ms, CUDA
+ * events around the main diagonal kernel only) and its launch count. */
+mp_status mp_last_timing(const mp_ctx* ctx, double* main_kernel_ms, int64_t* launches);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MP_H_ */

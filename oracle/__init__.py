@@ -40,7 +40,8 @@ def _load():
         lib.oracle_window_stats.argtypes = [p, i64, i64, i64, p, p]
         lib.oracle_cell.argtypes = [p, p, i64, i64, i64, i64, i64, p]
         lib.oracle_mstamp.argtypes = [p, p, i64, i64, i64, i64, p, i64, ctypes.c_int, p, p, p]
-        for f in (lib.oracle_window_stats, lib.oracle_cell, lib.oracle_mstamp):
+        lib.oracle_cells.argtypes = [p, p, i64, i64, i64, p, p, i64, p]
+        for f in (lib.oracle_window_stats, lib.oracle_cell, lib.oracle_mstamp, lib.oracle_cells):
             f.restype = ctypes.c_int
         _lib = lib
     return _lib
@@ -77,6 +78,20 @@ def cell(T, m, i, j, Tr=None):
     Tr_ = None if Tr is None else _series(Tr)
     out = np.empty(d)
     rc = _load().oracle_cell(_ptr(T), _ptr(Tr_), d, n, m, int(i), int(j), _ptr(out))
+    assert rc == 0
+    return out
+
+
+def cells(T, m, ii, jj, Tr=None):
+    """D''_k(ii[c], jj[c]) for all k: array (count, d)."""
+    T = _series(T)
+    d, L = T.shape
+    n = L - m + 1
+    Tr_ = None if Tr is None else _series(Tr)
+    ii = np.ascontiguousarray(ii, dtype=np.int64)
+    jj = np.ascontiguousarray(jj, dtype=np.int64)
+    out = np.empty((len(ii), d))
+    rc = _load().oracle_cells(_ptr(T), _ptr(Tr_), d, n, m, _ptr(ii), _ptr(jj), len(ii), _ptr(out))
     assert rc == 0
     return out
 

@@ -113,6 +113,28 @@ int oracle_cell(const double* Tq, const double* Tr, int64_t d, int64_t n, int64_
     return 0;
 }
 
+/* Many cells: out[c*d + k] = D''_k(ii[c], jj[c]); stats computed once. */
+int oracle_cells(const double* Tq, const double* Tr, int64_t d, int64_t n, int64_t m,
+                 const int64_t* ii, const int64_t* jj, int64_t count, double* out)
+{
+    if (!Tq || !ii || !jj || !out || d < 1 || n < 1 || m < 2 || count < 0) return 1;
+    for (int64_t c = 0; c < count; ++c)
+        if (ii[c] < 0 || ii[c] >= n || jj[c] < 0 || jj[c] >= n) return 1;
+    if (!Tr) Tr = Tq;
+    double* muq = malloc(sizeof(double) * d * n);
+    double* nq = malloc(sizeof(double) * d * n);
+    double* mur = malloc(sizeof(double) * d * n);
+    double* nr = malloc(sizeof(double) * d * n);
+    double* Db = malloc(sizeof(double) * d);
+    if (!muq || !nq || !mur || !nr || !Db) { free(muq); free(nq); free(mur); free(nr); free(Db); return 2; }
+    oracle_window_stats(Tq, d, n, m, muq, nq);
+    oracle_window_stats(Tr, d, n, m, mur, nr);
+    for (int64_t c = 0; c < count; ++c)
+        cell_dpp(Tq, Tr, d, n, m, muq, nq, mur, nr, ii[c], jj[c], Db, out + c * d);
+    free(muq); free(nq); free(mur); free(nr); free(Db);
+    return 0;
+}
+
 typedef struct {
     const double *Tq, *Tr, *muq, *nq, *mur, *nr;
     int64_t d, n, m, excl, self;

@@ -1,0 +1,391 @@
+// mp_api.cpp -- the C ABI (include/mp.h) and the host-side scheduler.
+//
+// Host responsibilities (the paper's Pseudocode 2 host driver, PAPER.md:L717-741,
+// re-designed): argument validation, the fixed tile plan (diagonal blocks x H-row
+// segments), the equal-cell diagonal-band partition across ranks (replaces the
+// paper's round-robin tile assignment, L709-712), device scratch caching, and the
+// launch sequence precompute -> fused diagonal kernel -> finalize.  All arithmetic of
+// the method runs in the CUDA kernels (mp_kernels.cu); nothing here computes on data.
+#include "../../include/mp.h"
+#include "mp_internal.h"
+
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+namespace {
+
+constexpr int64_t kDefaultH[4] = {4096, 1024, 256, 256};  // FP64, FP32, FP16, MIXED
+
+struct Buf {
+    void* p = nullptr;
+    size_t bytes = 0;
+};
+
+}  // namespace
+
+struct mp_ctx {
+    int device = 0;
+    int nsm = 148;
+    cudaStream_t stream = nullptr;
+    int64_t H[4] = {0, 0, 0, 0};
+    std::string err;
+    // cached scratch
+    Buf dT, dTr, st_q, st_r, tw_q, tw_r, mu_q, mu_r, nrm, keys, ext, seg, counter, dP, dI, flag;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    double last_ms = 0.0;
+    int64_t last_launches = 0;
+};
+
+namespace {
+
+mp_status fail(mp_ctx* ctx, mp_status st, const std::string& msg) {
+    if (ctx) ctx->err = msg;
+    return st;
+}
+
+mp_status cuda_fail(mp_ctx* ctx, cudaError_t e, const char* where) {
+    return fail(ctx, e == cudaErrorMemoryAllocation ? MP_ERR_NOMEM : MP_ERR_CUDA,
+                std::string(where) + ": " + cudaGetErrorString(e));
+}
+
+#define MP_CUDA(ctx, call)                                              \
+    do {                                                                \
+        cudaError_t e_ = (call);                                        \
+        if (e_ != cudaSuccess) return cuda_fail((ctx), e_, #call);      \
+    } while (0)
+
+cudaError_t ensure(Buf& b, size_t bytes) {
+    if (b.bytes >= bytes && b.p) return cudaSuccess;
+    if (b.p) cudaFree(b.p);
+    b.p = nullptr;
+    b.bytes = 0;
+    if (bytes == 0) bytes = 16;
+    cudaError_t e = cudaMalloc(&b.p, bytes);
+    if (e == cudaSuccess) b.bytes = bytes;
+    return e;
+}
+
+void release(Buf& b) {
+    if (b.p) cudaFree(b.p);
+    b.p = nullptr;
+    b.bytes = 0;
+}
+
+size_t elt_bytes(int prec) { return prec == MP_FP64 ? 8 : 4; }
+
+// ---------------------------------------------------------------- tile plan
+struct Plan {
+    int64_t dlo = 0, dhi = -1, nb = 0;
+    int nc = 32, H = 1024;
+    std::vector<long long> seg;    // nb + 1 exclusive prefix of segments
+    std::vector<double> cells;     // nb + 1 exclusive prefix of cells
+};
+
+Plan build_plan(int64_t d, int64_t n, int64_t excl, bool self, int prec, int64_t H) {
+    Plan pl;
+    pl.nc = mpk::pick_variant(prec, (int)d).NC;
+    pl.H = (int)H;
+    if (self) { pl.dlo = excl + 1; pl.dhi = n - 1; }
+    else { pl.dlo = -(n - 1); pl.dhi = n - 1; }
+    if (pl.dlo > pl.dhi) { pl.nb = 0; pl.seg.assign(1, 0); pl.cells.assign(1, 0.0); return pl; }
+    pl.nb = (pl.dhi - pl.dlo + 1 + pl.nc - 1) / pl.nc;
+    pl.seg.resize(pl.nb + 1);
+    pl.cells.resize(pl.nb + 1);
+    pl.seg[0] = 0;
+    pl.cells[0] = 0;
+    for (int64_t b = 0; b < pl.nb; ++b) {
+        const int64_t d0 = pl.dlo + b * pl.nc, d1 = std::min(d0 + pl.nc - 1, pl.dhi);
+        const int64_t rlo = std::max<int64_t>(0, -d1), rhi = std::min<int64_t>(n, n - std::max<int64_t>(d0, 0));
+        int64_t nseg = 0;
+        if (rlo < rhi) nseg = (rhi + H - 1) / H - rlo / H;
+        double c = 0;
+        for (int64_t dd = d0; dd <= d1; ++dd) c += (double)(n - (dd < 0 ? -dd : dd));
+        pl.seg[b + 1] = pl.seg[b] + nseg;
+        pl.cells[b + 1] = pl.cells[b] + c;
+    }
+    return pl;
+}
+
+// band g of world: blocks [bb[g], bb[g+1]) with (close to) equal cell counts
+std::vector<int64_t> band_blocks(const Plan& pl, int world) {
+    std::vector<int64_t> bb(world + 1, 0);
+    const double tot = pl.cells[pl.nb];
+    for (int g = 1; g < world; ++g) {
+        const double target = tot * g / world;
+        int64_t b = std::lower_bound(pl.cells.begin(), pl.cells.end(), target) - pl.cells.begin();
+        bb[g] = std::min<int64_t>(std::max<int64_t>(b, bb[g - 1]), pl.nb);
+    }
+    bb[world] = pl.nb;
+    return bb;
+}
+
+mp_status validate(mp_ctx* ctx, const void* T, int64_t d, int64_t n, int64_t m, int prec) {
+    if (!T) return fail(ctx, MP_ERR_INVALID, "T is NULL");
+    if (d < 1 || d > MP_MAX_D) return fail(ctx, MP_ERR_INVALID, "d must be in [1, 1024]");
+    if (n < 2) return fail(ctx, MP_ERR_INVALID, "n must be >= 2");
+    if (m < 2) return fail(ctx, MP_ERR_INVALID, "m must be >= 2");
+    if (n >= (int64_t(1) << 31) - 1) return fail(ctx, MP_ERR_INVALID, "n must be < 2^31");
+    if (m > (int64_t(1) << 20)) return fail(ctx, MP_ERR_INVALID, "m too large");
+    if (prec < 0 || prec > 3) return fail(ctx, MP_ERR_INVALID, "unknown precision");
+    if (prec == MP_FP16 || prec == MP_MIXED) return fail(ctx, MP_ERR_UNSUPPORTED, "FP16/MIXED not built yet");
+    if (prec == MP_FP64 && d > 512) return fail(ctx, MP_ERR_UNSUPPORTED, "FP64 supports d <= 512");
+    return MP_OK;
+}
+
+// Device pipeline: keys for band (rank, world) of the tile plan, internal key format.
+mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const double* dTr, int64_t d,
+                      int64_t n, int64_t m, int prec, int64_t excl, int rank, int world) {
+    const bool self = dTr == nullptr;
+    const int64_t L = n + m - 1;
+    const size_t eb = elt_bytes(prec);
+    const int64_t H = ctx->H[prec] > 0 ? ctx->H[prec] : kDefaultH[prec];
+    if (self && excl < 0) excl = (m + 3) / 4;
+
+    // flag non-finite inputs (reading G23)
+    MP_CUDA(ctx, ensure(ctx->flag, sizeof(int)));
+    MP_CUDA(ctx, cudaMemsetAsync(ctx->flag.p, 0, sizeof(int), s));
+    MP_CUDA(ctx, mpk::launch_check_finite(dT, d * L, (int*)ctx->flag.p, s));
+    if (!self) MP_CUDA(ctx, mpk::launch_check_finite(dTr, d * L, (int*)ctx->flag.p, s));
+    int flag = 0;
+    MP_CUDA(ctx, cudaMemcpyAsync(&flag, ctx->flag.p, sizeof(int), cudaMemcpyDeviceToHost, s));
+    MP_CUDA(ctx, cudaStreamSynchronize(s));
+    if (flag) return fail(ctx, MP_ERR_INVALID, "non-finite input");
+
+    // precalculation (Pseudocode 1 line 2)
+    MP_CUDA(ctx, ensure(ctx->st_q, (size_t)n * d * 4 * eb));
+    MP_CUDA(ctx, ensure(ctx->mu_q, (size_t)n * d * eb));
+    MP_CUDA(ctx, ensure(ctx->nrm, (size_t)n * d * eb));
+    if (prec != MP_FP64) MP_CUDA(ctx, ensure(ctx->tw_q, (size_t)L * d * eb));
+    mpk::PreParams pp{};
+    pp.n = n; pp.d = (int)d; pp.m = (int)m;
+    pp.nrm32 = (float*)ctx->nrm.p; pp.nrm64 = (double*)ctx->nrm.p;
+    pp.T = dT; pp.st = ctx->st_q.p; pp.mu = ctx->mu_q.p; pp.tw = ctx->tw_q.p;
+    MP_CUDA(ctx, mpk::launch_precompute(prec, pp, s));
+    if (!self) {
+        MP_CUDA(ctx, ensure(ctx->st_r, (size_t)n * d * 4 * eb));
+        MP_CUDA(ctx, ensure(ctx->mu_r, (size_t)n * d * eb));
+        if (prec != MP_FP64) MP_CUDA(ctx, ensure(ctx->tw_r, (size_t)L * d * eb));
+        pp.T = dTr; pp.st = ctx->st_r.p; pp.mu = ctx->mu_r.p; pp.tw = ctx->tw_r.p;
+        MP_CUDA(ctx, mpk::launch_precompute(prec, pp, s));
+    }
+
+    // keys
+    const size_t kb = (size_t)n * d * (prec == MP_FP64 ? 16 : 8);
+    MP_CUDA(ctx, ensure(ctx->keys, kb));
+    MP_CUDA(ctx, mpk::launch_init_keys(prec, ctx->keys.p, n * d, s));
+
+    // plan + band
+    Plan pl = build_plan(d, n, excl, self, prec, H);
+    ctx->last_launches = 0;
+    ctx->last_ms = 0.0;
+    if (pl.nb > 0) {
+        std::vector<int64_t> bb = band_blocks(pl, world);
+        const long long t_begin = pl.seg[bb[rank]], t_end = pl.seg[bb[rank + 1]];
+        MP_CUDA(ctx, ensure(ctx->seg, (pl.nb + 1) * sizeof(long long)));
+        MP_CUDA(ctx, cudaMemcpyAsync(ctx->seg.p, pl.seg.data(), (pl.nb + 1) * sizeof(long long),
+                                     cudaMemcpyHostToDevice, s));
+        MP_CUDA(ctx, ensure(ctx->counter, sizeof(unsigned long long)));
+        MP_CUDA(ctx, cudaMemsetAsync(ctx->counter.p, 0, sizeof(unsigned long long), s));
+        if (t_end > t_begin) {
+            mpk::MainParams mp{};
+            mp.st_q = ctx->st_q.p;
+            mp.st_r = self ? ctx->st_q.p : ctx->st_r.p;
+            mp.tw_q = prec == MP_FP64 ? (const void*)dT : ctx->tw_q.p;
+            mp.tw_r = self ? mp.tw_q : (prec == MP_FP64 ? (const void*)dTr : ctx->tw_r.p);
+            mp.mu_q = ctx->mu_q.p;
+            mp.mu_r = self ? ctx->mu_q.p : ctx->mu_r.p;
+            mp.keys = ctx->keys.p;
+            mp.seg_prefix = (const long long*)ctx->seg.p;
+            mp.nb = pl.nb;
+            mp.t_begin = t_begin;
+            mp.t_count = t_end - t_begin;
+            mp.counter = (unsigned long long*)ctx->counter.p;
+            mp.n = n; mp.d = (int)d; mp.m = (int)m; mp.H = (int)H;
+            mp.delta_lo = pl.dlo; mp.delta_hi = pl.dhi;
+            const int bps = std::max(1, mpk::main_blocks_per_sm(prec, (int)d, self));
+            const long long want_warps = mp.t_count;
+            long long grid = (long long)ctx->nsm * bps;
+            grid = std::min<long long>(grid, (want_warps + mpk::warps_per_block() - 1) / mpk::warps_per_block());
+            grid = std::max<long long>(grid, 1);
+            MP_CUDA(ctx, cudaEventRecord(ctx->ev0, s));
+            MP_CUDA(ctx, mpk::launch_main(prec, self, mp, (int)grid, s));
+            MP_CUDA(ctx, cudaEventRecord(ctx->ev1, s));
+            ctx->last_launches = 1;
+        }
+    }
+    return MP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* mp_version(void) { return "mstamp-b200 0.1 (sm_100a)"; }
+
+mp_status mp_init(mp_ctx** out, const mp_config* cfg) {
+    if (!out) return MP_ERR_INVALID;
+    *out = nullptr;
+    mp_ctx* ctx = new (std::nothrow) mp_ctx();
+    if (!ctx) return MP_ERR_NOMEM;
+    if (cfg) {
+        ctx->device = cfg->device;
+        for (int i = 0; i < 4; ++i) ctx->H[i] = cfg->reseed_h[i];
+    }
+    for (int i = 0; i < 4; ++i)
+        if (ctx->H[i] < 0) { delete ctx; return MP_ERR_INVALID; }
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev == 0) { delete ctx; return MP_ERR_CUDA; }
+    if (ctx->device < 0 || ctx->device >= ndev) { delete ctx; return MP_ERR_INVALID; }
+    if (cudaSetDevice(ctx->device) != cudaSuccess) { delete ctx; return MP_ERR_CUDA; }
+    cudaDeviceGetAttribute(&ctx->nsm, cudaDevAttrMultiProcessorCount, ctx->device);
+    if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreate(&ctx->ev0) != cudaSuccess || cudaEventCreate(&ctx->ev1) != cudaSuccess) {
+        mp_free(ctx);
+        return MP_ERR_CUDA;
+    }
+    *out = ctx;
+    return MP_OK;
+}
+
+void mp_free(mp_ctx* ctx) {
+    if (!ctx) return;
+    cudaSetDevice(ctx->device);
+    Buf* bufs[] = {&ctx->dT, &ctx->dTr, &ctx->st_q, &ctx->st_r, &ctx->tw_q, &ctx->tw_r, &ctx->mu_q,
+                   &ctx->mu_r, &ctx->nrm, &ctx->keys, &ctx->ext, &ctx->seg, &ctx->counter, &ctx->dP,
+                   &ctx->dI, &ctx->flag};
+    for (Buf* b : bufs) release(*b);
+    if (ctx->ev0) cudaEventDestroy(ctx->ev0);
+    if (ctx->ev1) cudaEventDestroy(ctx->ev1);
+    if (ctx->stream) cudaStreamDestroy(ctx->stream);
+    delete ctx;
+}
+
+const char* mp_last_error(const mp_ctx* ctx) {
+    if (!ctx) return "no context";
+    return ctx->err.c_str();
+}
+
+int64_t mp_key_words(int64_t d, int64_t n, mp_precision prec) {
+    return d * n * (prec == MP_FP64 ? 2 : 1);
+}
+
+mp_status mp_plan_bands(int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
+                        int self_join, int world, int64_t* block_begin, int64_t* cells) {
+    if (world < 1 || !block_begin || !cells || d < 1 || n < 2 || m < 2 || prec < 0 || prec > 3)
+        return MP_ERR_INVALID;
+    if (self_join && exclusion < 0) exclusion = (m + 3) / 4;
+    Plan pl = build_plan(d, n, exclusion, self_join != 0, prec, kDefaultH[prec]);
+    if (pl.nb == 0) {
+        for (int g = 0; g <= world; ++g) block_begin[g] = 0;
+        for (int g = 0; g < world; ++g) cells[g] = 0;
+        return MP_OK;
+    }
+    std::vector<int64_t> bb = band_blocks(pl, world);
+    for (int g = 0; g <= world; ++g) block_begin[g] = bb[g];
+    for (int g = 0; g < world; ++g) cells[g] = (int64_t)(pl.cells[bb[g + 1]] - pl.cells[bb[g]]);
+    return MP_OK;
+}
+
+mp_status mp_partial_device(mp_ctx* ctx, void* cuda_stream, const double* dT, const double* dTr,
+                            int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
+                            int rank, int world, int64_t* dKeys) {
+    if (!ctx) return MP_ERR_INVALID;
+    mp_status st = validate(ctx, dT, d, n, m, prec);
+    if (st != MP_OK) return st;
+    if (!dKeys || world < 1 || rank < 0 || rank >= world) return fail(ctx, MP_ERR_INVALID, "bad rank/world/keys");
+    MP_CUDA(ctx, cudaSetDevice(ctx->device));
+    cudaStream_t s = cuda_stream ? (cudaStream_t)cuda_stream : ctx->stream;
+    st = run_partial(ctx, s, dT, dTr, d, n, m, prec, exclusion, rank, world);
+    if (st != MP_OK) return st;
+    MP_CUDA(ctx, mpk::launch_keys_to_ext(prec, ctx->keys.p, dKeys, n * d, s));
+    return MP_OK;
+}
+
+mp_status mp_key_mask_device(mp_ctx* ctx, void* cuda_stream, int64_t d, int64_t n, int64_t* dKeys,
+                             const int64_t* dGlobalV) {
+    if (!ctx || !dKeys || !dGlobalV || d < 1 || n < 1) return fail(ctx, MP_ERR_INVALID, "bad arguments");
+    MP_CUDA(ctx, cudaSetDevice(ctx->device));
+    cudaStream_t s = cuda_stream ? (cudaStream_t)cuda_stream : ctx->stream;
+    MP_CUDA(ctx, mpk::launch_key_mask(n * d, (long long*)dKeys, (const long long*)dGlobalV, s));
+    return MP_OK;
+}
+
+mp_status mp_finalize_device(mp_ctx* ctx, void* cuda_stream, int64_t d, int64_t n, mp_precision prec,
+                             const int64_t* dKeys, double* dP, int64_t* dI) {
+    if (!ctx || !dKeys || !dP || !dI || d < 1 || n < 1) return fail(ctx, MP_ERR_INVALID, "bad arguments");
+    MP_CUDA(ctx, cudaSetDevice(ctx->device));
+    cudaStream_t s = cuda_stream ? (cudaStream_t)cuda_stream : ctx->stream;
+    MP_CUDA(ctx, mpk::launch_finalize(prec, dKeys, n, (int)d, dP, (long long*)dI, s));
+    return MP_OK;
+}
+
+mp_status mp_compute_device(mp_ctx* ctx, void* cuda_stream, const double* dT, const double* dTr,
+                            int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
+                            double* dP, int64_t* dI) {
+    if (!ctx) return MP_ERR_INVALID;
+    mp_status st = validate(ctx, dT, d, n, m, prec);
+    if (st != MP_OK) return st;
+    if (!dP || !dI) return fail(ctx, MP_ERR_INVALID, "P or I is NULL");
+    MP_CUDA(ctx, cudaSetDevice(ctx->device));
+    cudaStream_t s = cuda_stream ? (cudaStream_t)cuda_stream : ctx->stream;
+    st = run_partial(ctx, s, dT, dTr, d, n, m, prec, exclusion, 0, 1);
+    if (st != MP_OK) return st;
+    if (prec == MP_FP64) {
+        MP_CUDA(ctx, ensure(ctx->ext, (size_t)n * d * 16));
+        MP_CUDA(ctx, mpk::launch_keys_to_ext(prec, ctx->keys.p, ctx->ext.p, n * d, s));
+        MP_CUDA(ctx, mpk::launch_finalize(prec, ctx->ext.p, n, (int)d, dP, (long long*)dI, s));
+    } else {
+        MP_CUDA(ctx, mpk::launch_finalize(prec, ctx->keys.p, n, (int)d, dP, (long long*)dI, s));
+    }
+    return MP_OK;
+}
+
+mp_status mp_compute(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, int64_t n, int64_t m,
+                     mp_precision prec, int64_t exclusion, double* P, int64_t* I) {
+    if (!ctx) return MP_ERR_INVALID;
+    mp_status st = validate(ctx, T, d, n, m, prec);
+    if (st != MP_OK) return st;
+    if (!P || !I) return fail(ctx, MP_ERR_INVALID, "P or I is NULL");
+    const int64_t L = n + m - 1;
+    for (int64_t i = 0; i < d * L; ++i)
+        if (!std::isfinite(T[i]) || (Tr && !std::isfinite(Tr[i]))) return fail(ctx, MP_ERR_INVALID, "non-finite input");
+    MP_CUDA(ctx, cudaSetDevice(ctx->device));
+    cudaStream_t s = ctx->stream;
+    MP_CUDA(ctx, ensure(ctx->dT, (size_t)d * L * 8));
+    MP_CUDA(ctx, cudaMemcpyAsync(ctx->dT.p, T, (size_t)d * L * 8, cudaMemcpyHostToDevice, s));
+    if (Tr) {
+        MP_CUDA(ctx, ensure(ctx->dTr, (size_t)d * L * 8));
+        MP_CUDA(ctx, cudaMemcpyAsync(ctx->dTr.p, Tr, (size_t)d * L * 8, cudaMemcpyHostToDevice, s));
+    }
+    MP_CUDA(ctx, ensure(ctx->dP, (size_t)d * n * 8));
+    MP_CUDA(ctx, ensure(ctx->dI, (size_t)d * n * 8));
+    st = mp_compute_device(ctx, s, (const double*)ctx->dT.p, Tr ? (const double*)ctx->dTr.p : nullptr, d, n,
+                           m, prec, exclusion, (double*)ctx->dP.p, (int64_t*)ctx->dI.p);
+    if (st != MP_OK) return st;
+    MP_CUDA(ctx, cudaMemcpyAsync(P, ctx->dP.p, (size_t)d * n * 8, cudaMemcpyDeviceToHost, s));
+    MP_CUDA(ctx, cudaMemcpyAsync(I, ctx->dI.p, (size_t)d * n * 8, cudaMemcpyDeviceToHost, s));
+    MP_CUDA(ctx, cudaStreamSynchronize(s));
+    return MP_OK;
+}
+
+mp_status mp_last_timing(const mp_ctx* ctx, double* main_kernel_ms, int64_t* launches) {
+    if (!ctx || !main_kernel_ms || !launches) return MP_ERR_INVALID;
+    *launches = ctx->last_launches;
+    *main_kernel_ms = 0.0;
+    if (ctx->last_launches > 0) {
+        float ms = 0.f;
+        if (cudaEventSynchronize(ctx->ev1) != cudaSuccess) return MP_ERR_CUDA;
+        if (cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1) != cudaSuccess) return MP_ERR_CUDA;
+        *main_kernel_ms = ms;
+    }
+    return MP_OK;
+}
+
+}  // extern "C"

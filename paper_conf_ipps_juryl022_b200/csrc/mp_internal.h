@@ -1,0 +1,59 @@
+// Internal interface between the host scheduler (mp_api.cpp) and the CUDA kernels
+// (mp_kernels.cu).  Not part of the C ABI.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace mpk {
+
+// Parameters of the fused diagonal kernel (one launch = a contiguous tile range).
+struct MainParams {
+    const void* st_q;   // stats, position-major [pos][dim], V4 = (df, dg, a, 0)   (query / rows)
+    const void* st_r;   // stats of the reference series (columns); == st_q for self-join
+    const void* tw_q;   // working-precision series [dim][t], t < L (seeds)
+    const void* tw_r;
+    const void* mu_q;   // working-precision window means [dim][pos]
+    const void* mu_r;
+    void* keys;         // merge keys [pos][rank] of the QUERY profile (self-join: the one profile)
+    const long long* seg_prefix;  // exclusive prefix of #segments per diagonal block (NB+1)
+    long long nb;                 // number of diagonal blocks
+    long long t_begin, t_count;   // tile range of this launch
+    unsigned long long* counter;  // zeroed before launch
+    long long n;                  // subsequences
+    int d, m, H;                  // dims, window, re-seed interval (tile height)
+    long long delta_lo, delta_hi; // diagonal range [lo, hi] (j = i + delta)
+};
+
+struct PreParams {
+    const double* T;    // input [dim][t] FP64, L = n + m - 1
+    void* st;           // out stats [pos][dim]
+    void* tw;           // out working series [dim][t] (may alias nothing; FP64 mode: unused)
+    void* mu;           // out window mean [dim][pos]
+    float* nrm32;       // scratch for FP32 path (norm) [dim][pos]
+    double* nrm64;
+    long long n;
+    int d, m;
+};
+
+// Precision codes match mp_precision.
+enum { P64 = 0, P32 = 1, P16 = 2, PMIX = 3 };
+
+// Variant selection for a given (precision, d): dims per lane DL and lanes per cell G.
+struct Variant { int DL; int G; int NC; };
+Variant pick_variant(int prec, int d);
+size_t smem_per_block(int prec, int d, bool self);
+int warps_per_block();
+
+// Launchers (return cudaError_t).
+cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s);
+cudaError_t launch_init_keys(int prec, void* keys, long long count, cudaStream_t s);
+cudaError_t launch_main(int prec, bool self, const MainParams& p, int grid, cudaStream_t s);
+int main_blocks_per_sm(int prec, int d, bool self);
+cudaError_t launch_finalize(int prec, const void* keys_ext, long long n, int d, double* P,
+                            long long* I, cudaStream_t s);
+cudaError_t launch_keys_to_ext(int prec, const void* keys, void* ext, long long count,
+                               cudaStream_t s);
+cudaError_t launch_key_mask(long long count, long long* ext, const long long* gv, cudaStream_t s);
+cudaError_t launch_check_finite(const double* x, long long count, int* flag, cudaStream_t s);
+
+}  // namespace mpk

@@ -1,0 +1,215 @@
+// mp_kernels.cu -- precompute, key and finalize kernels + dispatch of the fused kernel.
+// The fused diagonal kernel itself lives in mp_diag.cuh (instantiated in inst_*.cu so
+// the heavy template variants compile in parallel).
+#include "mp_diag.cuh"
+
+namespace mpk {
+
+// ------------------------------------------------------------------ precompute
+// Per window (dim, pos): two-pass mean and norm in the precalc precision (Fig. 1 table,
+// L420-444), then df / dg (reading G7) and a = sqrt(2m)/norm (0 for flat windows, G4).
+template <class T>
+__global__ void pre_stats(const PreParams p) {
+    const long long n = p.n;
+    const int d = p.d, m = p.m;
+    const long long L = n + m - 1;
+    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (gid >= n * d) return;
+    const int dim = (int)(gid / n);
+    const long long pos = gid % n;
+    const double* x = p.T + (long long)dim * L + pos;
+    T s = 0;
+    for (int t = 0; t < m; ++t) s += (T)x[t];
+    const T mu = s / (T)m;
+    T q = 0;
+    for (int t = 0; t < m; ++t) {
+        const T cx = (T)x[t] - mu;
+        q = fma(cx, cx, q);
+    }
+    reinterpret_cast<T*>(p.mu)[(long long)dim * n + pos] = mu;
+    const T nr = sqrt(q);
+    if constexpr (sizeof(T) == 4) p.nrm32[(long long)dim * n + pos] = nr; else p.nrm64[(long long)dim * n + pos] = nr;
+}
+
+template <class T>
+__global__ void pre_diff(const PreParams p) {
+    using V4 = typename PT<T>::V4;
+    const long long n = p.n;
+    const int d = p.d, m = p.m;
+    const long long L = n + m - 1;
+    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (gid >= n * d) return;
+    const long long pos = gid / d;  // position-major output
+    const int dim = (int)(gid % d);
+    const double* x = p.T + (long long)dim * L;
+    const T* mu = reinterpret_cast<const T*>(p.mu) + (long long)dim * n;
+    T nr;
+    if constexpr (sizeof(T) == 4) nr = p.nrm32[(long long)dim * n + pos]; else nr = p.nrm64[(long long)dim * n + pos];
+    V4 v;
+    if (pos == 0) {
+        v.x = 0; v.y = 0;
+    } else {
+        const T xl = (T)x[pos + m - 1], xf = (T)x[pos - 1];
+        v.x = (xl - xf) / (T)2;
+        v.y = (xl - mu[pos]) + (xf - mu[pos - 1]);
+    }
+    v.z = nr > (T)0 ? sqrt((T)(2 * m)) / nr : (T)0;
+    v.w = 0;
+    reinterpret_cast<V4*>(p.st)[pos * d + dim] = v;
+}
+
+__global__ void to_f32(const double* x, float* y, long long count) {
+    const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i < count) y[i] = (float)x[i];
+}
+
+// ------------------------------------------------------------------ keys
+__global__ void init_keys32(unsigned long long* k, long long count) {
+    const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i < count) k[i] = EMPTY32;
+}
+__global__ void init_keys64(K64* k, long long count) {
+    const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i < count) { k[i].v = EMPTY64V; k[i].i = EMPTY64I; }
+}
+// FP64 AoS keys -> two int64 planes (value bits, index) for the collective merge
+__global__ void keys64_to_ext(const K64* k, long long* ext, long long count) {
+    const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i < count) {
+        ext[i] = (long long)k[i].v;
+        ext[count + i] = (k[i].v == EMPTY64V) ? (long long)EMPTY64I : (long long)k[i].i;
+    }
+}
+__global__ void key_mask(long long count, long long* ext, const long long* gv) {
+    const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i < count && ext[i] != gv[i]) ext[count + i] = (long long)EMPTY64I;
+}
+// ext keys [pos][rank] -> P [rank][pos] (sum / (k+1), reading G11), I [rank][pos]
+__global__ void finalize32(const unsigned long long* k, long long n, int d, double* P, long long* I) {
+    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (gid >= n * d) return;
+    const long long pos = gid / d;
+    const int rk = (int)(gid % d);
+    const unsigned long long key = k[gid];
+    double pv;
+    long long ix;
+    if (key >= EMPTY32) { pv = __longlong_as_double(0x7ff0000000000000ll); ix = -1; }
+    else { pv = (double)__uint_as_float((unsigned)(key >> 32)) / (double)(rk + 1); ix = (long long)(unsigned)key; }
+    P[(long long)rk * n + pos] = pv;
+    I[(long long)rk * n + pos] = ix;
+}
+__global__ void finalize64(const long long* ext, long long n, int d, double* P, long long* I) {
+    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    const long long count = n * d;
+    if (gid >= count) return;
+    const long long pos = gid / d;
+    const int rk = (int)(gid % d);
+    const unsigned long long v = (unsigned long long)ext[gid];
+    const long long ix = ext[count + gid];
+    double pv;
+    long long oi;
+    if (v >= EMPTY64V || ix == (long long)EMPTY64I) { pv = __longlong_as_double(0x7ff0000000000000ll); oi = -1; }
+    else { pv = __longlong_as_double((long long)v) / (double)(rk + 1); oi = ix; }
+    P[(long long)rk * n + pos] = pv;
+    I[(long long)rk * n + pos] = oi;
+}
+__global__ void check_finite(const double* x, long long count, int* flag) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < count;
+         i += (long long)gridDim.x * blockDim.x)
+        if (!isfinite(x[i])) atomicOr(flag, 1);
+}
+
+// ------------------------------------------------------------------ dispatch
+static inline unsigned grid1d(long long count, int bs) { return (unsigned)((count + bs - 1) / bs); }
+
+Variant pick_variant(int prec, int d) {
+    // FP32: a lane holds up to 32 dims; FP64: up to 16 (register budget).
+    const int maxdl = prec == P64 ? 16 : 32;
+    int dp = 1;
+    while (dp < d) dp <<= 1;
+    Variant v;
+    if (dp <= maxdl) { v.DL = dp; v.G = 1; }
+    else { v.DL = maxdl; v.G = dp / maxdl; }
+    v.NC = 32 / v.G;
+    return v;
+}
+
+int warps_per_block() { return WARPS_PER_BLOCK; }
+
+// op: 0 = smem, 1 = launch, 2 = blocks/SM
+template <class T, bool SELF>
+static long long dispatch_t(int op, int DL, int G, const MainParams* p, int grid, cudaStream_t s) {
+#define MP_CASE(dl, g)                                                                 \
+    if (DL == dl && G == g) {                                                          \
+        if (op == 0) return (long long)Inst<T, dl, g, SELF>::smem();                   \
+        if (op == 1) return (long long)Inst<T, dl, g, SELF>::launch(*p, grid, s);      \
+        return Inst<T, dl, g, SELF>::blocks_per_sm();                                  \
+    }
+    MP_CASE(1, 1) MP_CASE(2, 1) MP_CASE(4, 1) MP_CASE(8, 1) MP_CASE(16, 1)
+    if constexpr (sizeof(T) == 4) { MP_CASE(32, 1) MP_CASE(32, 2) MP_CASE(32, 4) MP_CASE(32, 8) MP_CASE(32, 16) MP_CASE(32, 32) }
+    else { MP_CASE(16, 2) MP_CASE(16, 4) MP_CASE(16, 8) MP_CASE(16, 16) MP_CASE(16, 32) }
+#undef MP_CASE
+    return op == 1 ? (long long)cudaErrorInvalidValue : 0;
+}
+
+static long long dispatch(int op, int prec, bool self, int d, const MainParams* p, int grid, cudaStream_t s) {
+    const Variant v = pick_variant(prec, d);
+    if (prec == P64) return self ? dispatch_t<double, true>(op, v.DL, v.G, p, grid, s) : dispatch_t<double, false>(op, v.DL, v.G, p, grid, s);
+    if (prec == P32) return self ? dispatch_t<float, true>(op, v.DL, v.G, p, grid, s) : dispatch_t<float, false>(op, v.DL, v.G, p, grid, s);
+    return op == 1 ? (long long)cudaErrorInvalidValue : 0;
+}
+
+size_t smem_per_block(int prec, int d, bool self) { return (size_t)dispatch(0, prec, self, d, nullptr, 0, 0); }
+int main_blocks_per_sm(int prec, int d, bool self) { return (int)dispatch(2, prec, self, d, nullptr, 0, 0); }
+cudaError_t launch_main(int prec, bool self, const MainParams& p, int grid, cudaStream_t s) {
+    return (cudaError_t)dispatch(1, prec, self, p.d, &p, grid, s);
+}
+
+cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s) {
+    const long long cnt = p.n * p.d;
+    const long long L = p.n + p.m - 1;
+    if (prec == P64) {
+        pre_stats<double><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+        pre_diff<double><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+    } else if (prec == P32) {
+        pre_stats<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+        pre_diff<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+        to_f32<<<grid1d(L * p.d, 256), 256, 0, s>>>(p.T, reinterpret_cast<float*>(p.tw), L * p.d);
+    } else {
+        return cudaErrorInvalidValue;
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_init_keys(int prec, void* keys, long long count, cudaStream_t s) {
+    if (prec == P64) init_keys64<<<grid1d(count, 256), 256, 0, s>>>(reinterpret_cast<K64*>(keys), count);
+    else init_keys32<<<grid1d(count, 256), 256, 0, s>>>(reinterpret_cast<unsigned long long*>(keys), count);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_keys_to_ext(int prec, const void* keys, void* ext, long long count, cudaStream_t s) {
+    if (prec == P64) {
+        keys64_to_ext<<<grid1d(count, 256), 256, 0, s>>>(reinterpret_cast<const K64*>(keys), reinterpret_cast<long long*>(ext), count);
+        return cudaGetLastError();
+    }
+    return cudaMemcpyAsync(ext, keys, count * sizeof(long long), cudaMemcpyDeviceToDevice, s);
+}
+
+cudaError_t launch_key_mask(long long count, long long* ext, const long long* gv, cudaStream_t s) {
+    key_mask<<<grid1d(count, 256), 256, 0, s>>>(count, ext, gv);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_finalize(int prec, const void* keys_ext, long long n, int d, double* P, long long* I, cudaStream_t s) {
+    const long long cnt = n * d;
+    if (prec == P64) finalize64<<<grid1d(cnt, 256), 256, 0, s>>>(reinterpret_cast<const long long*>(keys_ext), n, d, P, I);
+    else finalize32<<<grid1d(cnt, 256), 256, 0, s>>>(reinterpret_cast<const unsigned long long*>(keys_ext), n, d, P, I);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_check_finite(const double* x, long long count, int* flag, cudaStream_t s) {
+    check_finite<<<1184, 256, 0, s>>>(x, count, flag);
+    return cudaGetLastError();
+}
+
+}  // namespace mpk

@@ -1,0 +1,221 @@
+"""Thin ctypes binding of libmstamp_b200.so (include/mp.h).
+
+Argument marshalling only: every step of the method runs in the CUDA kernels
+behind the C ABI.  There is no CPU fallback -- ``load()`` raises if the shared
+library is missing or no CUDA device is usable.
+
+Host-memory entry point: ``Context.compute(T, m, ...)`` (numpy in/out, includes
+the H2D/D2H copies).  Device entry points take torch CUDA tensors (torch is used
+only for device memory, streams and process groups).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "lib", "libmstamp_b200.so")
+
+PRECISIONS = {"fp64": 0, "fp32": 1, "fp16": 2, "mixed": 3}
+STATUS = {0: "MP_OK", 1: "MP_ERR_INVALID", 2: "MP_ERR_NOMEM", 3: "MP_ERR_CUDA", 4: "MP_ERR_NCCL",
+          5: "MP_ERR_UNSUPPORTED"}
+EXPORTS = ["mp_init", "mp_free", "mp_last_error", "mp_version", "mp_compute", "mp_compute_device",
+           "mp_key_words", "mp_partial_device", "mp_key_mask_device", "mp_finalize_device",
+           "mp_plan_bands", "mp_last_timing"]
+
+_lib = None
+
+
+class MPError(RuntimeError):
+    def __init__(self, status, msg=""):
+        self.status = status
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+
+
+class _Config(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int), ("reseed_h", ctypes.c_int64 * 4)]
+
+
+def load():
+    """Load the C-ABI library (fails loudly if it was not built)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise RuntimeError(f"{LIB_PATH} missing: run __graft_entry__.build() (no CPU fallback exists)")
+    lib = ctypes.CDLL(LIB_PATH)
+    i64, p, i32 = ctypes.c_int64, ctypes.c_void_p, ctypes.c_int
+    lib.mp_init.argtypes = [ctypes.POINTER(p), ctypes.POINTER(_Config)]
+    lib.mp_init.restype = i32
+    lib.mp_free.argtypes = [p]
+    lib.mp_free.restype = None
+    lib.mp_last_error.argtypes = [p]
+    lib.mp_last_error.restype = ctypes.c_char_p
+    lib.mp_version.argtypes = []
+    lib.mp_version.restype = ctypes.c_char_p
+    lib.mp_compute.argtypes = [p, p, p, i64, i64, i64, i32, i64, p, p]
+    lib.mp_compute.restype = i32
+    lib.mp_compute_device.argtypes = [p, p, p, p, i64, i64, i64, i32, i64, p, p]
+    lib.mp_compute_device.restype = i32
+    lib.mp_key_words.argtypes = [i64, i64, i32]
+    lib.mp_key_words.restype = i64
+    lib.mp_partial_device.argtypes = [p, p, p, p, i64, i64, i64, i32, i64, i32, i32, p]
+    lib.mp_partial_device.restype = i32
+    lib.mp_key_mask_device.argtypes = [p, p, i64, i64, p, p]
+    lib.mp_key_mask_device.restype = i32
+    lib.mp_finalize_device.argtypes = [p, p, i64, i64, i32, p, p, p]
+    lib.mp_finalize_device.restype = i32
+    lib.mp_plan_bands.argtypes = [i64, i64, i64, i32, i64, i32, i32, p, p]
+    lib.mp_plan_bands.restype = i32
+    lib.mp_last_timing.argtypes = [p, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(i64)]
+    lib.mp_last_timing.restype = i32
+    _lib = lib
+    return lib
+
+
+def _prec(prec):
+    if isinstance(prec, str):
+        return PRECISIONS[prec.lower()]
+    return int(prec)
+
+
+def version() -> str:
+    return load().mp_version().decode()
+
+
+def plan_bands(d, n, m, prec="fp32", exclusion=-1, self_join=True, world=1):
+    """Host scheduler: (block_begin[world+1], cells[world]) of the equal-cell diagonal bands."""
+    lib = load()
+    bb = np.zeros(world + 1, dtype=np.int64)
+    cells = np.zeros(world, dtype=np.int64)
+    st = lib.mp_plan_bands(d, n, m, _prec(prec), exclusion, int(bool(self_join)), world,
+                           bb.ctypes.data_as(ctypes.c_void_p), cells.ctypes.data_as(ctypes.c_void_p))
+    if st != 0:
+        raise MPError(st, "mp_plan_bands")
+    return bb, cells
+
+
+def key_words(d, n, prec="fp32") -> int:
+    return int(load().mp_key_words(d, n, _prec(prec)))
+
+
+def _tptr(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+class Context:
+    """One context per host thread / GPU (mp_init ... mp_free)."""
+
+    def __init__(self, device: int = 0, reseed_h=None):
+        lib = load()
+        cfg = _Config()
+        cfg.device = device
+        h = list(reseed_h or [0, 0, 0, 0])
+        for i in range(4):
+            cfg.reseed_h[i] = int(h[i])
+        self._ctx = ctypes.c_void_p()
+        st = lib.mp_init(ctypes.byref(self._ctx), ctypes.byref(cfg))
+        if st != 0:
+            raise MPError(st, "mp_init")
+        self.device = device
+
+    def close(self):
+        if self._ctx:
+            load().mp_free(self._ctx)
+            self._ctx = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def _check(self, st, what):
+        if st != 0:
+            raise MPError(st, f"{what}: {load().mp_last_error(self._ctx).decode()}")
+
+    # ---- host memory
+    def compute(self, T, m, prec="fp32", exclusion=-1, Tr=None):
+        """P (d,n) float64 and I (d,n) int64 from host series T (d,L) [and Tr]."""
+        T = np.ascontiguousarray(T, dtype=np.float64)
+        if T.ndim == 1:
+            T = T[None, :]
+        d, L = T.shape
+        n = L - m + 1
+        Tr_ = None
+        if Tr is not None:
+            Tr_ = np.ascontiguousarray(Tr, dtype=np.float64)
+            if Tr_.ndim == 1:
+                Tr_ = Tr_[None, :]
+            if Tr_.shape != T.shape:
+                raise MPError(1, "AB-join needs equal shapes")
+        P = np.empty((d, n), dtype=np.float64)
+        I = np.empty((d, n), dtype=np.int64)
+        st = load().mp_compute(self._ctx, T.ctypes.data_as(ctypes.c_void_p),
+                               None if Tr_ is None else Tr_.ctypes.data_as(ctypes.c_void_p),
+                               d, n, m, _prec(prec), int(exclusion),
+                               P.ctypes.data_as(ctypes.c_void_p), I.ctypes.data_as(ctypes.c_void_p))
+        self._check(st, "mp_compute")
+        return P, I
+
+    # ---- device memory (torch tensors)
+    def compute_device(self, T, m, P, I, prec="fp32", exclusion=-1, Tr=None, stream=None):
+        import torch
+        d, L = T.shape
+        n = L - m + 1
+        s = stream if stream is not None else torch.cuda.current_stream(T.device)
+        st = load().mp_compute_device(self._ctx, ctypes.c_void_p(s.cuda_stream), _tptr(T), _tptr(Tr),
+                                      d, n, m, _prec(prec), int(exclusion), _tptr(P), _tptr(I))
+        self._check(st, "mp_compute_device")
+
+    def partial_device(self, T, m, keys, rank, world, prec="fp32", exclusion=-1, Tr=None, stream=None):
+        import torch
+        d, L = T.shape
+        n = L - m + 1
+        s = stream if stream is not None else torch.cuda.current_stream(T.device)
+        st = load().mp_partial_device(self._ctx, ctypes.c_void_p(s.cuda_stream), _tptr(T), _tptr(Tr),
+                                      d, n, m, _prec(prec), int(exclusion), int(rank), int(world),
+                                      _tptr(keys))
+        self._check(st, "mp_partial_device")
+
+    def key_mask_device(self, d, n, keys, global_v, stream=None):
+        import torch
+        s = stream if stream is not None else torch.cuda.current_stream(keys.device)
+        st = load().mp_key_mask_device(self._ctx, ctypes.c_void_p(s.cuda_stream), d, n, _tptr(keys),
+                                       _tptr(global_v))
+        self._check(st, "mp_key_mask_device")
+
+    def finalize_device(self, d, n, keys, P, I, prec="fp32", stream=None):
+        import torch
+        s = stream if stream is not None else torch.cuda.current_stream(keys.device)
+        st = load().mp_finalize_device(self._ctx, ctypes.c_void_p(s.cuda_stream), d, n, _prec(prec),
+                                       _tptr(keys), _tptr(P), _tptr(I))
+        self._check(st, "mp_finalize_device")
+
+    def last_timing(self):
+        ms = ctypes.c_double()
+        nl = ctypes.c_int64()
+        self._check(load().mp_last_timing(self._ctx, ctypes.byref(ms), ctypes.byref(nl)), "mp_last_timing")
+        return ms.value, nl.value
+
+
+def merge_partials(ctx: Context, keys, d, n, prec, group=None):
+    """MINLOC all-reduce of partial keys over the process group (the path's one exchange).
+
+    FP32/FP16/MIXED: one int64 MIN.  FP64: MIN on the value plane, mask indices whose
+    value lost, MIN on the index plane.  ``keys`` is modified in place.
+    """
+    import torch.distributed as dist
+    count = d * n
+    if _prec(prec) == 0:
+        v = keys[:count]
+        gv = v.clone()
+        dist.all_reduce(gv, op=dist.ReduceOp.MIN, group=group)
+        ctx.key_mask_device(d, n, keys, gv)
+        v.copy_(gv)
+        dist.all_reduce(keys[count:], op=dist.ReduceOp.MIN, group=group)
+    else:
+        dist.all_reduce(keys, op=dist.ReduceOp.MIN, group=group)
+    return keys

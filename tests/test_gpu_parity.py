@@ -1,0 +1,187 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the FP64 oracle, element by element.
+
+Marked gpu; the oracle is test infrastructure and never on the product path.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import parity
+from paper_conf_ipps_juryl022_b200 import datagen
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ipps_juryl022_b200 import mstamp
+    c = mstamp.Context(0)
+    yield c
+    c.close()
+
+
+@pytest.fixture(scope="module")
+def c1_oracle(oracle_mod):
+    cfg = datagen.make("C1")
+    P, I, P2 = oracle_mod.mstamp(cfg["T"], cfg["m"], cfg["exclusion"])
+    return cfg, P, I, P2
+
+
+@pytest.mark.parametrize("prec", ["fp64", "fp32"])
+def test_c1_full(ctx, oracle_mod, c1_oracle, prec):
+    """BASELINE config C1 (d=4, n=4096, m=64, planted motif), every (k, i)."""
+    cfg, P, I, P2 = c1_oracle
+    Pg, Ig = ctx.compute(cfg["T"], cfg["m"], prec, cfg["exclusion"])
+    st = parity.check(oracle_mod, cfg["T"], cfg["m"], P, I, P2, Pg, Ig, prec)
+    print(prec, st)
+    a, b = datagen.motif_positions(cfg["n"], cfg["m"])
+    for k in range(max(1, cfg["d"] // 2)):
+        assert Ig[k, a] == b and Ig[k, b] == a
+
+
+SHAPES = [  # (d, n, m, exclusion, seed): ragged tails, several tiles, odd d, tiny n
+    (1, 300, 8, 2, 1), (2, 77, 5, 1, 2), (3, 1500, 16, 4, 3), (5, 700, 32, 8, 4),
+    (8, 2100, 12, 3, 5), (16, 1100, 64, 16, 6), (17, 600, 16, 4, 7), (32, 400, 8, 2, 8),
+    (33, 300, 10, 3, 9), (64, 250, 16, 4, 10), (100, 200, 8, 2, 11), (7, 5000, 24, 6, 12),
+]
+
+
+@pytest.mark.parametrize("prec", ["fp64", "fp32"])
+@pytest.mark.parametrize("shape", SHAPES)
+def test_random_shapes_self(ctx, oracle_mod, prec, shape):
+    d, n, m, e, seed = shape
+    if prec == "fp64" and d > 512:
+        pytest.skip()
+    T = datagen.random_walk(d, n, m, seed)
+    P, I, P2 = oracle_mod.mstamp(T, m, e)
+    Pg, Ig = ctx.compute(T, m, prec, e)
+    parity.check(oracle_mod, T, m, P, I, P2, Pg, Ig, prec)
+
+
+@pytest.mark.parametrize("prec", ["fp64", "fp32"])
+@pytest.mark.parametrize("shape", [(1, 200, 8, 21), (4, 900, 16, 22), (16, 500, 32, 23), (40, 150, 8, 24)])
+def test_random_shapes_ab(ctx, oracle_mod, prec, shape):
+    d, n, m, seed = shape
+    Tq, Tr = datagen.random_walk_ab(d, n, m, seed)
+    P, I, P2 = oracle_mod.mstamp(Tq, m, Tr=Tr)
+    Pg, Ig = ctx.compute(Tq, m, prec, Tr=Tr)
+    parity.check(oracle_mod, Tq, m, P, I, P2, Pg, Ig, prec, Tr=Tr)
+
+
+def test_golden_m2(ctx):
+    """Hand-derived closed-form profile (tests/golden/m2_selfjoin.txt) on the GPU, FP64."""
+    import test_oracle
+    T, meta, rows = test_oracle._read_golden("m2_selfjoin.txt")
+    for prec in ("fp64", "fp32"):
+        Pg, Ig = ctx.compute(T, meta["m"], prec, meta["exclusion"])
+        for (i, k, p, ok) in rows:
+            assert abs(Pg[k, i] - p) < 1e-3, (prec, i, k, Pg[k, i], p)
+            assert int(Ig[k, i]) in ok, (prec, i, k, Ig[k, i], ok)
+
+
+@pytest.mark.parametrize("prec", ["fp64", "fp32"])
+def test_exclusion_edge(ctx, oracle_mod, prec):
+    """Reading G3: everything excluded -> P = inf, I = -1; nearly everything excluded."""
+    T = datagen.random_walk(3, 40, 8, 31)
+    Pg, Ig = ctx.compute(T, 8, prec, 39)
+    assert np.all(np.isinf(Pg)) and np.all(Ig == -1)
+    P, I, P2 = oracle_mod.mstamp(T, 8, 37)
+    Pg, Ig = ctx.compute(T, 8, prec, 37)
+    parity.check(oracle_mod, T, 8, P, I, P2, Pg, Ig, prec)
+
+
+def test_flat_windows(ctx, oracle_mod):
+    """Reading G4 on the GPU: constant windows (norm 0) -> rho = 0."""
+    T = datagen.random_walk(2, 400, 16, 32)
+    T[0, 100:160] = 3.0
+    P, I, P2 = oracle_mod.mstamp(T, 16, 4)
+    Pg, Ig = ctx.compute(T, 16, "fp64", 4)
+    parity.check(oracle_mod, T, 16, P, I, P2, Pg, Ig, "fp64")
+
+
+@pytest.mark.parametrize("prec", ["fp64", "fp32"])
+def test_reseed_interval_independent(ctx, oracle_mod, prec):
+    """Re-seed interval H changes the recurrence's rounding path but not the result (within tol)."""
+    from paper_conf_ipps_juryl022_b200 import mstamp
+    T = datagen.random_walk(4, 3000, 32, 33)
+    P, I, P2 = oracle_mod.mstamp(T, 32, 8)
+    for h in (7, 64, 5000):
+        c = mstamp.Context(0, reseed_h=[h, h, h, h])
+        Pg, Ig = c.compute(T, 32, prec, 8)
+        c.close()
+        parity.check(oracle_mod, T, 32, P, I, P2, Pg, Ig, prec)
+
+
+@pytest.mark.parametrize("prec", ["fp64", "fp32"])
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_bands_bit_identical(ctx, prec, world):
+    """Band partition emulated on one GPU: per-rank partial keys merged by MIN (the NCCL
+    collective's semantics) are bit-identical to the single-band result."""
+    from paper_conf_ipps_juryl022_b200 import mstamp
+    d, n, m = 6, 3000, 32
+    T = torch.from_numpy(datagen.random_walk(d, n, m, 34)).cuda()
+    cnt = d * n
+    kw = mstamp.key_words(d, n, prec)
+    full = torch.empty(kw, dtype=torch.int64, device="cuda")
+    ctx.partial_device(T, m, full, 0, 1, prec, 8)
+    parts = []
+    for r in range(world):
+        k = torch.empty(kw, dtype=torch.int64, device="cuda")
+        ctx.partial_device(T, m, k, r, world, prec, 8)
+        parts.append(k)
+    st = torch.stack(parts)
+    if prec == "fp64":
+        gv = st[:, :cnt].min(dim=0).values
+        for k in parts:
+            ctx.key_mask_device(d, n, k, gv)
+        merged = torch.cat([gv, torch.stack(parts)[:, cnt:].min(dim=0).values])
+    else:
+        merged = st.min(dim=0).values
+    torch.cuda.synchronize()
+    assert torch.equal(merged, full)
+    P1 = torch.empty(d, n, dtype=torch.float64, device="cuda")
+    I1 = torch.empty(d, n, dtype=torch.int64, device="cuda")
+    ctx.finalize_device(d, n, merged, P1, I1, prec)
+    Pd = torch.empty_like(P1)
+    Id = torch.empty_like(I1)
+    ctx.compute_device(T, m, Pd, Id, prec, 8)
+    torch.cuda.synchronize()
+    assert torch.equal(P1, Pd) and torch.equal(I1, Id)
+
+
+@pytest.mark.parametrize("prec", ["fp64", "fp32"])
+def test_c2_sampled_rows(ctx, oracle_mod, prec):
+    """BASELINE config C2 at full size (d=16, n=65536, m=128) in the bench's launch
+    configuration; sampled query rows checked one by one against the oracle."""
+    cfg = datagen.make("C2")
+    T, m, e, n = cfg["T"], cfg["m"], cfg["exclusion"], cfg["n"]
+    Pg, Ig = ctx.compute(T, m, prec, e)
+    a, b = datagen.motif_positions(n, m)
+    rows = np.unique(np.concatenate([[0, 1, n - 1, n - 2, a, b], np.random.default_rng(5).integers(0, n, 20)]))
+    P, I, P2 = oracle_mod.mstamp(T, m, e, rows=rows)
+    st = parity.check(oracle_mod, T, m, P, I, P2, Pg, Ig, prec, rows=rows)
+    print(prec, st)
+    # properties at every (k, i): bound, monotone in k, symmetry P[I] <= P (self-join)
+    assert np.all(Pg >= 0) and np.all(Pg <= 2 * math.sqrt(m) * (1 + 1e-6))
+    assert np.all(np.diff(Pg, axis=0) >= -1e-6 * Pg[1:])
+    for k in (0, 7, 15):
+        assert np.all(Pg[k, Ig[k]] <= Pg[k] * (1 + 1e-6) + 1e-6)
+
+
+def test_invalid_arguments(ctx):
+    from paper_conf_ipps_juryl022_b200 import mstamp
+    T = datagen.random_walk(2, 50, 8, 1)
+    bad = T.copy()
+    bad[1, 3] = np.nan
+    with pytest.raises(mstamp.MPError) as ei:
+        ctx.compute(bad, 8, "fp32")
+    assert ei.value.status == 1
+    with pytest.raises(mstamp.MPError):
+        ctx.compute(T, 1, "fp32")
+    with pytest.raises(mstamp.MPError):
+        ctx.compute(np.zeros((2000, 10)), 4, "fp32")
