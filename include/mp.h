@@ -88,7 +88,8 @@ mp_status mp_compute(mp_ctx* ctx, const double* T, const double* Tr,
                      int64_t d, int64_t n, int64_t m, mp_precision prec,
                      int64_t exclusion, double* P, int64_t* I);
 
-/* Same as mp_compute with DEVICE pointers on the caller's CUDA stream (may be NULL). */
+/* Same as mp_compute with DEVICE pointers, enqueued on the caller's CUDA stream (NULL = the
+ * legacy default stream).  Returns after enqueueing (one host sync for the input check). */
 mp_status mp_compute_device(mp_ctx* ctx, void* cuda_stream, const double* dT, const double* dTr,
                             int64_t d, int64_t n, int64_t m, mp_precision prec,
                             int64_t exclusion, double* dP, int64_t* dI);
@@ -106,7 +107,7 @@ mp_status mp_compute_device(mp_ctx* ctx, void* cuda_stream, const double* dT, co
  *                      reduce with MIN over int64.
  *     FP64: two int64 planes; plane 0 = double bits of the distance SUM (reduce MIN),
  *           plane 1 = index; call mp_key_mask_device between the two MIN reductions.
- *   Empty entries are INT64_MAX.
+ *   Empty entries: FP32 keys >= 0x7F80000000000000 (value +inf); FP64 index plane INT64_MAX.
  */
 int64_t   mp_key_words(int64_t d, int64_t n, mp_precision prec);
 mp_status mp_partial_device(mp_ctx* ctx, void* cuda_stream, const double* dT, const double* dTr,

@@ -3,5 +3,7 @@
 #define MP_DIAG_IMPL
 #include "mp_diag.cuh"
 namespace mpk {
-template struct Inst<float, 16, 1, 1, false>;
+template struct Inst<float, 1, 1, 2, true>;
+template struct Inst<float, 2, 1, 2, true>;
+template struct Inst<float, 4, 1, 2, true>;
 }  // namespace mpk

@@ -1,6 +1,7 @@
-// generated by build layout: explicit instantiations of the fused diagonal kernel
+// Explicit instantiations of the fused diagonal kernel (split across translation units
+// so the template variants compile in parallel; see build.py).
 #define MP_DIAG_IMPL
 #include "mp_diag.cuh"
 namespace mpk {
-template struct Inst<double, 16, 1, false>;
+template struct Inst<double, 16, 1, 1, false>;
 }  // namespace mpk

@@ -3,5 +3,5 @@
 #define MP_DIAG_IMPL
 #include "mp_diag.cuh"
 namespace mpk {
-template struct Inst<float, 16, 1, 1, false>;
+template struct Inst<double, 16, 8, 1, false>;
 }  // namespace mpk

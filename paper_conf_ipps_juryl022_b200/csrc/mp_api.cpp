@@ -20,7 +20,16 @@
 
 namespace {
 
-constexpr int64_t kDefaultH[4] = {4096, 1024, 256, 256};  // FP64, FP32, FP16, MIXED
+constexpr int64_t kDefaultH[4] = {4096, 1024, 256, 256};  // FP64, FP32, FP16, MIXED (upper bounds)
+
+// Default re-seed interval H (= tile height, the paper's tiling lever against error growth,
+// PAPER.md:L700-703).  The recurrence error grows with H relative to the window energy, which
+// scales with m, so reduced precisions re-seed every 8m rows (seed cost m/H stays 1/8 of a
+// cell-dim's recurrence work), capped by the per-precision maximum.
+int64_t default_h(int prec, int64_t m) {
+    if (prec == MP_FP64) return kDefaultH[prec];
+    return std::max<int64_t>(64, std::min<int64_t>(kDefaultH[prec], 8 * m));
+}
 
 struct Buf {
     void* p = nullptr;
@@ -36,7 +45,7 @@ struct mp_ctx {
     int64_t H[4] = {0, 0, 0, 0};
     std::string err;
     // cached scratch
-    Buf dT, dTr, st_q, st_r, tw_q, tw_r, mu_q, mu_r, nrm, keys, ext, seg, counter, dP, dI, flag;
+    Buf dT, dTr, st_q, st_r, tw_q, tw_r, mu_q, mu_r, mup_q, mup_r, nrm, keys, ext, seg, counter, dP, dI, flag;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     double last_ms = 0.0;
     int64_t last_launches = 0;
@@ -144,7 +153,7 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     const bool self = dTr == nullptr;
     const int64_t L = n + m - 1;
     const size_t eb = elt_bytes(prec);
-    const int64_t H = ctx->H[prec] > 0 ? ctx->H[prec] : kDefaultH[prec];
+    const int64_t H = ctx->H[prec] > 0 ? ctx->H[prec] : default_h(prec, m);
     if (self && excl < 0) excl = (m + 3) / 4;
 
     // flag non-finite inputs (reading G23)
@@ -159,19 +168,23 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
 
     // precalculation (Pseudocode 1 line 2)
     MP_CUDA(ctx, ensure(ctx->st_q, (size_t)n * d * 4 * eb));
+    const mpk::Variant var = mpk::pick_variant(prec, (int)d);
+    const int Dp = var.DL * var.G;
     MP_CUDA(ctx, ensure(ctx->mu_q, (size_t)n * d * eb));
+    MP_CUDA(ctx, ensure(ctx->mup_q, (size_t)n * Dp * eb));
     MP_CUDA(ctx, ensure(ctx->nrm, (size_t)n * d * eb));
-    if (prec != MP_FP64) MP_CUDA(ctx, ensure(ctx->tw_q, (size_t)L * d * eb));
+    MP_CUDA(ctx, ensure(ctx->tw_q, (size_t)L * Dp * eb));
     mpk::PreParams pp{};
-    pp.n = n; pp.d = (int)d; pp.m = (int)m;
+    pp.n = n; pp.d = (int)d; pp.m = (int)m; pp.Dp = Dp;
     pp.nrm32 = (float*)ctx->nrm.p; pp.nrm64 = (double*)ctx->nrm.p;
-    pp.T = dT; pp.st = ctx->st_q.p; pp.mu = ctx->mu_q.p; pp.tw = ctx->tw_q.p;
+    pp.T = dT; pp.st = ctx->st_q.p; pp.mu = ctx->mu_q.p; pp.tw = ctx->tw_q.p; pp.mup = ctx->mup_q.p;
     MP_CUDA(ctx, mpk::launch_precompute(prec, pp, s));
     if (!self) {
         MP_CUDA(ctx, ensure(ctx->st_r, (size_t)n * d * 4 * eb));
         MP_CUDA(ctx, ensure(ctx->mu_r, (size_t)n * d * eb));
-        if (prec != MP_FP64) MP_CUDA(ctx, ensure(ctx->tw_r, (size_t)L * d * eb));
-        pp.T = dTr; pp.st = ctx->st_r.p; pp.mu = ctx->mu_r.p; pp.tw = ctx->tw_r.p;
+        MP_CUDA(ctx, ensure(ctx->mup_r, (size_t)n * Dp * eb));
+        MP_CUDA(ctx, ensure(ctx->tw_r, (size_t)L * Dp * eb));
+        pp.T = dTr; pp.st = ctx->st_r.p; pp.mu = ctx->mu_r.p; pp.tw = ctx->tw_r.p; pp.mup = ctx->mup_r.p;
         MP_CUDA(ctx, mpk::launch_precompute(prec, pp, s));
     }
 
@@ -196,10 +209,10 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
             mpk::MainParams mp{};
             mp.st_q = ctx->st_q.p;
             mp.st_r = self ? ctx->st_q.p : ctx->st_r.p;
-            mp.tw_q = prec == MP_FP64 ? (const void*)dT : ctx->tw_q.p;
-            mp.tw_r = self ? mp.tw_q : (prec == MP_FP64 ? (const void*)dTr : ctx->tw_r.p);
-            mp.mu_q = ctx->mu_q.p;
-            mp.mu_r = self ? ctx->mu_q.p : ctx->mu_r.p;
+            mp.tw_q = ctx->tw_q.p;
+            mp.tw_r = self ? ctx->tw_q.p : ctx->tw_r.p;
+            mp.mu_q = ctx->mup_q.p;
+            mp.mu_r = self ? ctx->mup_q.p : ctx->mup_r.p;
             mp.keys = ctx->keys.p;
             mp.seg_prefix = (const long long*)ctx->seg.p;
             mp.nb = pl.nb;
@@ -211,7 +224,8 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
             const int bps = std::max(1, mpk::main_blocks_per_sm(prec, (int)d, self));
             const long long want_warps = mp.t_count;
             long long grid = (long long)ctx->nsm * bps;
-            grid = std::min<long long>(grid, (want_warps + mpk::warps_per_block() - 1) / mpk::warps_per_block());
+            const int wpb = std::max(1, mpk::variant_warps_per_block(prec, (int)d, self));
+            grid = std::min<long long>(grid, (want_warps + wpb - 1) / wpb);
             grid = std::max<long long>(grid, 1);
             MP_CUDA(ctx, cudaEventRecord(ctx->ev0, s));
             MP_CUDA(ctx, mpk::launch_main(prec, self, mp, (int)grid, s));
@@ -258,7 +272,7 @@ void mp_free(mp_ctx* ctx) {
     if (!ctx) return;
     cudaSetDevice(ctx->device);
     Buf* bufs[] = {&ctx->dT, &ctx->dTr, &ctx->st_q, &ctx->st_r, &ctx->tw_q, &ctx->tw_r, &ctx->mu_q,
-                   &ctx->mu_r, &ctx->nrm, &ctx->keys, &ctx->ext, &ctx->seg, &ctx->counter, &ctx->dP,
+                   &ctx->mu_r, &ctx->mup_q, &ctx->mup_r, &ctx->nrm, &ctx->keys, &ctx->ext, &ctx->seg, &ctx->counter, &ctx->dP,
                    &ctx->dI, &ctx->flag};
     for (Buf* b : bufs) release(*b);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
@@ -281,7 +295,7 @@ mp_status mp_plan_bands(int64_t d, int64_t n, int64_t m, mp_precision prec, int6
     if (world < 1 || !block_begin || !cells || d < 1 || n < 2 || m < 2 || prec < 0 || prec > 3)
         return MP_ERR_INVALID;
     if (self_join && exclusion < 0) exclusion = (m + 3) / 4;
-    Plan pl = build_plan(d, n, exclusion, self_join != 0, prec, kDefaultH[prec]);
+    Plan pl = build_plan(d, n, exclusion, self_join != 0, prec, default_h(prec, m));
     if (pl.nb == 0) {
         for (int g = 0; g <= world; ++g) block_begin[g] = 0;
         for (int g = 0; g < world; ++g) cells[g] = 0;
@@ -301,7 +315,7 @@ mp_status mp_partial_device(mp_ctx* ctx, void* cuda_stream, const double* dT, co
     if (st != MP_OK) return st;
     if (!dKeys || world < 1 || rank < 0 || rank >= world) return fail(ctx, MP_ERR_INVALID, "bad rank/world/keys");
     MP_CUDA(ctx, cudaSetDevice(ctx->device));
-    cudaStream_t s = cuda_stream ? (cudaStream_t)cuda_stream : ctx->stream;
+    cudaStream_t s = (cudaStream_t)cuda_stream;  // NULL = the legacy default stream
     st = run_partial(ctx, s, dT, dTr, d, n, m, prec, exclusion, rank, world);
     if (st != MP_OK) return st;
     MP_CUDA(ctx, mpk::launch_keys_to_ext(prec, ctx->keys.p, dKeys, n * d, s));
@@ -312,7 +326,7 @@ mp_status mp_key_mask_device(mp_ctx* ctx, void* cuda_stream, int64_t d, int64_t 
                              const int64_t* dGlobalV) {
     if (!ctx || !dKeys || !dGlobalV || d < 1 || n < 1) return fail(ctx, MP_ERR_INVALID, "bad arguments");
     MP_CUDA(ctx, cudaSetDevice(ctx->device));
-    cudaStream_t s = cuda_stream ? (cudaStream_t)cuda_stream : ctx->stream;
+    cudaStream_t s = (cudaStream_t)cuda_stream;  // NULL = the legacy default stream
     MP_CUDA(ctx, mpk::launch_key_mask(n * d, (long long*)dKeys, (const long long*)dGlobalV, s));
     return MP_OK;
 }
@@ -321,7 +335,7 @@ mp_status mp_finalize_device(mp_ctx* ctx, void* cuda_stream, int64_t d, int64_t 
                              const int64_t* dKeys, double* dP, int64_t* dI) {
     if (!ctx || !dKeys || !dP || !dI || d < 1 || n < 1) return fail(ctx, MP_ERR_INVALID, "bad arguments");
     MP_CUDA(ctx, cudaSetDevice(ctx->device));
-    cudaStream_t s = cuda_stream ? (cudaStream_t)cuda_stream : ctx->stream;
+    cudaStream_t s = (cudaStream_t)cuda_stream;  // NULL = the legacy default stream
     MP_CUDA(ctx, mpk::launch_finalize(prec, dKeys, n, (int)d, dP, (long long*)dI, s));
     return MP_OK;
 }
@@ -334,7 +348,7 @@ mp_status mp_compute_device(mp_ctx* ctx, void* cuda_stream, const double* dT, co
     if (st != MP_OK) return st;
     if (!dP || !dI) return fail(ctx, MP_ERR_INVALID, "P or I is NULL");
     MP_CUDA(ctx, cudaSetDevice(ctx->device));
-    cudaStream_t s = cuda_stream ? (cudaStream_t)cuda_stream : ctx->stream;
+    cudaStream_t s = (cudaStream_t)cuda_stream;  // NULL = the legacy default stream
     st = run_partial(ctx, s, dT, dTr, d, n, m, prec, exclusion, 0, 1);
     if (st != MP_OK) return st;
     if (prec == MP_FP64) {

@@ -15,11 +15,12 @@
 //
 // Execution model (B200-first, not the paper's 3-kernels-per-row loop):
 //   one warp owns a tile of NC consecutive diagonals x H rows; G lanes cooperate on a
-//   cell when d > 32 (each holds DL dims); the NC cells of a warp step are arranged as
-//   RA rows x CA columns (row = r0 + s - CA*a, col = row + delta) so a step touches
-//   RA distinct rows and CA distinct columns.  Row/column statistics and the running
-//   profile thresholds are staged in per-warp shared-memory rings (rows enter once per
-//   step, leave after RA*CA steps), so the inner loop reads 2 LDS per cell-dim.  The
+//   cell when d > 32 (each holds DL dims), and for small d a lane owns W = 2 adjacent
+//   diagonals (same row, columns j and j+1; column j+1's data is carried in registers to
+//   the next step, halving shared-memory traffic).  The lane-cells of a warp step are
+//   arranged as RA rows x CA columns (row = r0 + s - CA*W*a) so a step touches RA rows
+//   and CA*W columns.  Row/column statistics and the running profile thresholds are
+//   staged in per-warp shared-memory rings by cp.async (LDGSTS) one step ahead.  The
 //   profile update is filtered: a cell only does work if some S_k <= current best of
 //   its row or column (fresh per warp, seeded from global memory at row entry); such
 //   steps run a warp-shuffle group-min + leader update, and dirty rows/columns are
@@ -30,6 +31,9 @@
 #include <cstdint>
 #include <cmath>
 #include "mp_internal.h"
+#ifndef MP_MINB
+#define MP_MINB 1
+#endif
 
 namespace mpk {
 
@@ -69,21 +73,55 @@ template <class T> __device__ __forceinline__ void cswap(T& a, T& b) {
     b = hi;
 }
 
-// Batcher odd-even merge sort network on N registers (any N; fully unrolled at compile
-// time).  Ascending (Eq. 2 "sort", reading G12).
+// Ampere-style async global->shared copies (LDGSTS): ring staging without registers.
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(sa), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(sa), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async4(void* smem, const void* gmem) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(sa), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
+
+// Batcher odd-even merge sort network on N registers (any N), ascending (Eq. 2 "sort",
+// PAPER.md:L642-643, reading G12).  The comparator list is generated at compile time
+// (constexpr) so every register index is a constant after unrolling.
+constexpr int batcher_count(int N) {
+    int c = 0;
+    for (int p = 1; p < N; p <<= 1)
+        for (int k = p; k >= 1; k >>= 1)
+            for (int j = k % p; j + k < N; j += 2 * k)
+                for (int i = 0; i < k; ++i)
+                    if (i + j + k < N && (i + j) / (2 * p) == (i + j + k) / (2 * p)) ++c;
+    return c;
+}
+template <int N> struct BatcherNet {
+    static constexpr int C = batcher_count(N) > 0 ? batcher_count(N) : 1;
+    short a[C], b[C];
+    constexpr BatcherNet() : a{}, b{} {
+        int c = 0;
+        for (int p = 1; p < N; p <<= 1)
+            for (int k = p; k >= 1; k >>= 1)
+                for (int j = k % p; j + k < N; j += 2 * k)
+                    for (int i = 0; i < k; ++i)
+                        if (i + j + k < N && (i + j) / (2 * p) == (i + j + k) / (2 * p)) {
+                            a[c] = (short)(i + j);
+                            b[c] = (short)(i + j + k);
+                            ++c;
+                        }
+    }
+};
 template <class T, int N> __device__ __forceinline__ void sort_net(T (&v)[N]) {
+    if constexpr (N > 1) {
+        constexpr BatcherNet<N> net{};
 #pragma unroll
-    for (int p = 1; p < N; p <<= 1) {
-#pragma unroll
-        for (int k = p; k >= 1; k >>= 1) {
-#pragma unroll
-            for (int j = k % p; j + k < N; j += 2 * k) {
-#pragma unroll
-                for (int i = 0; i < k; ++i) {
-                    if (i + j + k < N && (i + j) / (2 * p) == (i + j + k) / (2 * p)) cswap(v[i + j], v[i + j + k]);
-                }
-            }
-        }
+        for (int c = 0; c < batcher_count(N); ++c) cswap(v[net.a[c]], v[net.b[c]]);
     }
 }
 
@@ -130,17 +168,19 @@ template <class T, int DL, int G> __device__ __forceinline__ void lane_merge(T (
 // FP32: key = (float bits of S << 32) | j   (non-negative floats are order-isomorphic
 //       to their bits, so u64 min == lexicographic (value, index) min, reading G2).
 // FP64: {double bits of S, j} compared lexicographically, merged by 128-bit CAS.
-constexpr unsigned long long EMPTY32 = 0x7F800000FFFFFFFFull;          // (+inf, 2^32-1)
+// Empty entries carry index 0x7FFFFFFF so a staged index never has the DIRTY bit.
+constexpr unsigned long long EMPTY32 = 0x7F8000007FFFFFFFull;          // (+inf, 2^31-1)
 constexpr unsigned long long EMPTY64V = 0x7FF0000000000000ull;         // +inf
-constexpr unsigned long long EMPTY64I = 0x7FFFFFFFFFFFFFFFull;
+constexpr unsigned long long EMPTY64I = 0x000000007FFFFFFFull;
+constexpr long long EXT_EMPTY = 0x7FFFFFFFFFFFFFFFll;                  // INT64_MAX (ABI)
 
 template <class T> struct KeyOps;
 template <> struct KeyOps<float> {
     using K = unsigned long long;
-    static __device__ __forceinline__ void load(const K* p, float& v, unsigned& i) {
-        K k = __ldcg(p);
-        v = __uint_as_float((unsigned)(k >> 32));
-        i = (unsigned)k;
+    // async-stage the key's value (high word) into thr and its index (low word) into idx
+    static __device__ __forceinline__ void stage(const K* p, float* thr, unsigned* idx) {
+        cp_async4(thr, reinterpret_cast<const char*>(p) + 4);
+        cp_async4(idx, p);
     }
     static __device__ __forceinline__ void merge(K* p, float v, unsigned i) {
         atomicMin(p, ((K)__float_as_uint(v) << 32) | (K)i);
@@ -149,10 +189,9 @@ template <> struct KeyOps<float> {
 struct alignas(16) K64 { unsigned long long v, i; };
 template <> struct KeyOps<double> {
     using K = K64;
-    static __device__ __forceinline__ void load(const K* p, double& v, unsigned& i) {
-        ulonglong2 k = __ldcg(reinterpret_cast<const ulonglong2*>(p));
-        v = __longlong_as_double((long long)k.x);
-        i = (k.y > 0xffffffffull) ? 0xffffffffu : (unsigned)k.y;
+    static __device__ __forceinline__ void stage(const K* p, double* thr, unsigned* idx) {
+        cp_async8(thr, &p->v);
+        cp_async4(idx, &p->i);  // little-endian low word; indices < 2^31
     }
     static __device__ __forceinline__ void merge(K* p, double v, unsigned i) {
         unsigned long long nv = (unsigned long long)__double_as_longlong(v), ni = i;
@@ -172,35 +211,66 @@ template <> struct KeyOps<double> {
     }
 };
 
+// Load the DL dims a lane owns (dims kk*G + g) of one position-major, D-padded row.
+template <class T, int DL, int G>
+__device__ __forceinline__ void load_dims(const T* __restrict__ rowp, int g, T (&out)[DL]) {
+    if constexpr (G == 1 && sizeof(T) == 4 && DL % 4 == 0) {
+#pragma unroll
+        for (int q = 0; q < DL / 4; ++q) {
+            const float4 v = __ldg(reinterpret_cast<const float4*>(rowp) + q);
+            out[4 * q] = v.x; out[4 * q + 1] = v.y; out[4 * q + 2] = v.z; out[4 * q + 3] = v.w;
+        }
+    } else if constexpr (G == 1 && sizeof(T) == 8 && DL % 2 == 0) {
+#pragma unroll
+        for (int q = 0; q < DL / 2; ++q) {
+            const double2 v = __ldg(reinterpret_cast<const double2*>(rowp) + q);
+            out[2 * q] = v.x; out[2 * q + 1] = v.y;
+        }
+    } else {
+#pragma unroll
+        for (int kk = 0; kk < DL; ++kk) out[kk] = __ldg(rowp + kk * G + g);
+    }
+}
+
 // ------------------------------------------------------------------ tile geometry
-template <int G> struct Geo {
-    static constexpr int NC = 32 / G;                                   // cells per warp step
-    static constexpr int CA = NC >= 16 ? 4 : (NC >= 4 ? 2 : 1);         // distinct columns per step
-    static constexpr int RA = NC / CA;                                   // distinct rows per step
-    static constexpr int LIVE_R = CA * (RA - 1) + 2;
-    static constexpr int RING_R0 = LIVE_R <= 2 ? 2 : LIVE_R <= 4 ? 4 : LIVE_R <= 8 ? 8 : LIVE_R <= 16 ? 16 : 32;
-    static constexpr int RING_R = RING_R0 < 8 ? 8 : RING_R0;
-    static constexpr int RPC = RING_R / CA;                              // ring rows per residue class
-    static constexpr int RING_C = (2 * CA) < 8 ? 8 : 2 * CA;
-    static constexpr int PSR = RING_R + RA;                              // plane stride (elements), padded
-    static constexpr int PSC = RING_C + CA;
-    static constexpr int LOG_G = G == 1 ? 0 : G == 2 ? 1 : G == 4 ? 2 : G == 8 ? 3 : G == 16 ? 4 : 5;
-    static constexpr int LOG_CA = CA == 1 ? 0 : CA == 2 ? 1 : 2;
-    // ring slot of row r: rows spaced CA apart land in consecutive slots of one class
+constexpr int pow2ceil(int x) { int p = 1; while (p < x) p <<= 1; return p; }
+constexpr int ilog2(int x) { int l = 0; while ((1 << l) < x) ++l; return l; }
+
+template <int G, int W> struct Geo {
+    static constexpr int NL = 32 / G;                                   // lane-cells per warp
+    static constexpr int CA = NL >= 16 ? 4 : (NL >= 4 ? 2 : 1);         // lane-cells per row group
+    static constexpr int RA = NL / CA;                                   // distinct rows per step
+    static constexpr int CW = CA * W;                                    // distinct columns per step
+    static constexpr int NC = NL * W;                                    // cells (diagonals) per warp
+    // ring positions move in batches of SB steps, prefetched one batch ahead: live rows
+    // span CW(RA-1) + 2 SB, live columns 2 SB + CW - 1
+    static constexpr int SB = 2;
+    static constexpr int RING_R = pow2ceil(CW * (RA - 1) + 2 * SB) < CW ? CW : pow2ceil(CW * (RA - 1) + 2 * SB);
+    static constexpr int RPC = RING_R / CW;                              // ring rows per residue class
+    static constexpr int RING_C = pow2ceil(2 * SB + CW - 1);
+    // plane strides (V4 units): odd for G == 1 so the planes of an entering position hit
+    // distinct banks; for G > 1 the G planes read together are shifted by RA (CW) slots.
+    static constexpr int PSR = G == 1 ? RING_R + 1 : RING_R + RA;
+    static constexpr int PSC = G == 1 ? RING_C + 1 : RING_C + CW;
+    static constexpr int LOG_G = ilog2(G), LOG_CA = ilog2(CA), LOG_CW = ilog2(CW), LOG_RPC = ilog2(RPC);
+    // ring slot of row r: rows spaced CW apart land in consecutive slots of one class
     static __device__ __forceinline__ int srow(long long r) {
-        int ri = (int)r;
-        return (ri & (CA - 1)) * RPC + ((ri >> LOG_CA) & (RPC - 1));
+        const int ri = (int)r;
+        return ((ri & (CW - 1)) << LOG_RPC) + ((ri >> LOG_CW) & (RPC - 1));
     }
     static __device__ __forceinline__ int scol(long long c) { return (int)c & (RING_C - 1); }
 };
 
-template <class T, int DL, int G> struct Smem {
+template <class T, int DL, int G, int W> struct Smem {
     using V4 = typename PT<T>::V4;
-    using Gm = Geo<G>;
+    using Gm = Geo<G, W>;
     static constexpr int D = DL * G;
     static constexpr size_t ring_bytes =
         (((size_t)D * (Gm::PSR + Gm::PSC) * (sizeof(V4) + sizeof(unsigned))) + 15) & ~(size_t)15;
-    static constexpr size_t bytes_per_warp = ring_bytes + (size_t)DL * 32 * sizeof(T);  // + slow-path scratch
+    static constexpr size_t flag_bytes = ((Gm::RING_R + Gm::RING_C) * 4 + 15) & ~(size_t)15;
+    static constexpr size_t bytes_per_warp = ring_bytes + flag_bytes + (size_t)W * DL * 32 * sizeof(T);
+    // warps per block: up to 4, fewer when a warp's rings are large (blocks <= ~112 KB)
+    static constexpr int WPB = bytes_per_warp * 4 <= 112 * 1024 ? 4 : bytes_per_warp * 2 <= 112 * 1024 ? 2 : 1;
 };
 
 // plane p holds dimension p's stats in .xyz and, in .w, the threshold of rank
@@ -208,24 +278,33 @@ template <class T, int DL, int G> struct Smem {
 template <int DL, int G> __device__ __forceinline__ int rank_of_plane(int p) { return (p % G) * DL + p / G; }
 
 // ------------------------------------------------------------------ the fused kernel
-template <class T, int DL, int G, bool SELF>
-__global__ void __launch_bounds__(WARPS_PER_BLOCK * 32)
+// minimum resident blocks per SM for the register budget (128 threads per block max)
+template <class T, int DL, int G, int W> constexpr int min_blocks() {
+    // caps the register budget where ptxas still fits without spills (measured with -Xptxas -v)
+    return (sizeof(T) == 4 && G == 1 && DL * W <= 16) ? 3 : MP_MINB;
+}
+template <class T, int DL, int G, int W, bool SELF>
+__global__ void __launch_bounds__(128, (min_blocks<T, DL, G, W>()))
 mp_diag(const MainParams p) {
     using V4 = typename PT<T>::V4;
-    using Gm = Geo<G>;
+    using Gm = Geo<G, W>;
+    using SM = Smem<T, DL, G, W>;
     using KO = KeyOps<T>;
     using K = typename KO::K;
-    constexpr int NC = Gm::NC, CA = Gm::CA, RA = Gm::RA, D = DL * G;
+    constexpr int CA = Gm::CA, RA = Gm::RA, CW = Gm::CW, D = DL * G;
     constexpr int PSR = Gm::PSR, PSC = Gm::PSC;
+    constexpr int SB = Gm::SB;
 
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    unsigned char* wbase = smem_raw + (size_t)warp * Smem<T, DL, G>::bytes_per_warp;
+    unsigned char* wbase = smem_raw + (size_t)warp * SM::bytes_per_warp;
     V4* rowv = reinterpret_cast<V4*>(wbase);
     V4* colv = rowv + (size_t)D * PSR;
     unsigned* rowi = reinterpret_cast<unsigned*>(colv + (size_t)D * PSC);
     unsigned* coli = rowi + (size_t)D * PSR;
-    T* ssc = reinterpret_cast<T*>(wbase + Smem<T, DL, G>::ring_bytes);
+    unsigned* rowdirty = reinterpret_cast<unsigned*>(wbase + SM::ring_bytes);
+    unsigned* coldirty = rowdirty + Gm::RING_R;
+    T* ssc = reinterpret_cast<T*>(wbase + SM::ring_bytes + SM::flag_bytes);
 
     const V4* __restrict__ st_q = reinterpret_cast<const V4*>(p.st_q);
     const V4* __restrict__ st_r = reinterpret_cast<const V4*>(p.st_r);
@@ -241,55 +320,83 @@ mp_diag(const MainParams p) {
     const T two_m = (T)(2 * m);
     const T INF = PT<T>::inf(), NINF = PT<T>::ninf();
 
-    const int cell = lane >> Gm::LOG_G, g = lane & (G - 1);
-    const int a = cell >> Gm::LOG_CA, c = cell & (CA - 1);
-    // lanes of the same row group (same a, g): vary c; same column group (c, g): vary a
-    const unsigned gmask_row = [&] {
-        unsigned mk = 0;
-        for (int cc = 0; cc < CA; ++cc) mk |= 1u << (((a * CA + cc) << Gm::LOG_G) + g);
-        return mk;
-    }();
-    const unsigned gmask_col = [&] {
-        unsigned mk = 0;
-        for (int aa = 0; aa < RA; ++aa) mk |= 1u << (((aa * CA + c) << Gm::LOG_G) + g);
-        return mk;
-    }();
+    const int lc = lane >> Gm::LOG_G, g = lane & (G - 1);
+    const int a = lc >> Gm::LOG_CA, c = lc & (CA - 1);
+    // lanes of the same row group (same a, g) vary c; same column group (c, g) vary a
+    unsigned gmask_row = 0, gmask_col = 0;
+#pragma unroll
+    for (int cc = 0; cc < CA; ++cc) gmask_row |= 1u << (((a * CA + cc) << Gm::LOG_G) + g);
+#pragma unroll
+    for (int aa = 0; aa < RA; ++aa) gmask_col |= 1u << (((aa * CA + c) << Gm::LOG_G) + g);
 
-    // --- ring staging helpers (each lane handles planes lane, lane+32, ...)
-    auto enter = [&](bool is_row, long long pos, const V4* __restrict__ st) {
-        if (pos < 0 || pos >= n) return;
+    // --- ring staging.  Positions move through the rings in batches of SB steps:
+    // stage() starts the async copies (cp.async / LDGSTS) of a range of entering positions'
+    // stats (.xyz), thresholds (.w = the value half of the merge key) and best indices one
+    // batch ahead; evict() merges positions whose ring copy improved (dirty) into global
+    // memory.  The (position, plane) pairs of a range are spread over the 32 lanes.
+    const int n32 = (int)n;
+    auto stage = [&](bool is_row, int base, int p_lo, int p_hi) {
+        const int cnt = p_hi - p_lo;
+        if (cnt <= 0) return;
         V4* buf = is_row ? rowv : colv;
         unsigned* ib = is_row ? rowi : coli;
+        unsigned* dflag = is_row ? rowdirty : coldirty;
         const int ps = is_row ? PSR : PSC;
-        const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
-        for (int pl = lane; pl < D; pl += 32) {
-            V4 v;
+        const V4* __restrict__ st = is_row ? st_q : st_r;
+        const bool want_thr = is_row || SELF;
+        for (int e = lane; e < cnt * D; e += 32) {
+            const int pi = e / D, pl = e - pi * D;
+            const int pos = base + p_lo + pi;
+            if (pos < 0 || pos >= n32) continue;
+            const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
+            if (pl == 0) dflag[sl] = 0;
+            V4* dst = &buf[pl * ps + sl];
+            const V4* src = st + (size_t)pos * d + pl;
             if (pl < d) {
-                v = st[pos * d + pl];
+                if constexpr (sizeof(T) == 4) {
+                    cp_async8(dst, src);                      // df, dg
+                    cp_async4(&dst->z, &src->z);              // a
+                } else {
+                    cp_async16(dst, src);
+                    cp_async8(&dst->z, &src->z);
+                }
             } else {  // padded dimension: a = +inf with QT = -1 gives D = +inf (sorts last)
-                v.x = 0; v.y = 0; v.z = INF;
+                dst->x = 0; dst->y = 0; dst->z = INF;
             }
             const int rk = rank_of_plane<DL, G>(pl);
-            unsigned ix = 0;
-            T thr = NINF;  // never hit
-            if (rk < d && (is_row || SELF)) KO::load(keys + pos * d + rk, thr, ix);
-            v.w = thr;
-            buf[pl * ps + sl] = v;
-            ib[pl * ps + sl] = ix & ~DIRTY;
+            if (rk < d && want_thr) {
+                KO::stage(keys + (size_t)pos * d + rk, &dst->w, &ib[pl * ps + sl]);
+            } else {
+                dst->w = NINF;  // never hit
+                ib[pl * ps + sl] = 0x7fffffffu;
+            }
         }
     };
-    auto leave = [&](bool is_row, long long pos) {
-        if (pos < 0 || pos >= n) return;
+    auto evict = [&](bool is_row, int base, int p_lo, int p_hi) {
         if (!is_row && !SELF) return;
+        const int cnt = p_hi - p_lo;
+        if (cnt <= 0) return;
         const V4* buf = is_row ? rowv : colv;
         const unsigned* ib = is_row ? rowi : coli;
+        const unsigned* dflag = is_row ? rowdirty : coldirty;
         const int ps = is_row ? PSR : PSC;
-        const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
-        for (int pl = lane; pl < D; pl += 32) {
+        // early out: most evictions find nothing dirty
+        bool any = false;
+        for (int pi = lane; pi < cnt; pi += 32) {
+            const int pos = base + p_lo + pi;
+            if (pos >= 0 && pos < n32) any |= dflag[is_row ? Gm::srow(pos) : Gm::scol(pos)] != 0;
+        }
+        if (!__any_sync(FULL, any)) return;
+        for (int e = lane; e < cnt * D; e += 32) {
+            const int pi = e / D, pl = e - pi * D;
+            const int pos = base + p_lo + pi;
+            if (pos < 0 || pos >= n32) continue;
+            const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
+            if (dflag[sl] == 0) continue;
             const int rk = rank_of_plane<DL, G>(pl);
             if (rk >= d) continue;
             const unsigned ix = ib[pl * ps + sl];
-            if (ix & DIRTY) KO::merge(keys + pos * d + rk, buf[pl * ps + sl].w, ix & ~DIRTY);
+            if (ix & DIRTY) KO::merge(keys + (size_t)pos * d + rk, buf[pl * ps + sl].w, ix & ~DIRTY);
         }
     };
 
@@ -302,183 +409,295 @@ mp_diag(const MainParams p) {
         // block b: seg_prefix[b] <= t < seg_prefix[b+1]
         long long lo_b = 0, hi_b = p.nb;
         while (hi_b - lo_b > 1) {
-            long long mid = (lo_b + hi_b) >> 1;
-            if (p.seg_prefix[mid] <= t) lo_b = mid; else hi_b = mid;
+            const long long mid = (lo_b + hi_b) >> 1;
+            if (__ldg(&p.seg_prefix[mid]) <= t) lo_b = mid; else hi_b = mid;
         }
         const long long b = lo_b;
-        const long long delta0 = p.delta_lo + b * NC;
-        const long long delta1 = min(delta0 + NC - 1, p.delta_hi);
+        const long long delta0 = p.delta_lo + b * Gm::NC;
+        const long long delta1 = min(delta0 + Gm::NC - 1, p.delta_hi);
         const long long rlo = max(0ll, -delta1), rhi = min(n, n - max(delta0, 0ll));
-        const long long q = rlo / H + (t - p.seg_prefix[b]);
+        const long long q = rlo / H + (t - __ldg(&p.seg_prefix[b]));
         const long long r0 = max(q * H, rlo), r1 = min((q + 1) * H, rhi);
 
-        // lane's diagonal and its valid row range inside the tile
-        const long long delta = delta0 + cell;
-        long long lo = max(r0, max(0ll, -delta));
-        long long hi = min(r1, n - max(delta, 0ll));
-        if (delta > p.delta_hi) hi = lo;
-
-        // seeds: direct centred dot products at row lo (reading G8)
-        T QT[DL];
+        // the lane's W cells: diagonals and valid row ranges inside the tile
+        long long delta[W], lo[W], hi[W];
 #pragma unroll
-        for (int kk = 0; kk < DL; ++kk) {
-            const int dim = kk * G + g;
-            T acc = (T)0;
-            if (dim >= d) {
-                acc = (T)-1;
-            } else if (lo < hi) {
-                const T* xq = tw_q + (long long)dim * L + lo;
-                const T* xr = tw_r + (long long)dim * L + lo + delta;
-                const T mq = mu_q[(long long)dim * n + lo], mr = mu_r[(long long)dim * n + lo + delta];
-                for (int tt = 0; tt < m; ++tt) acc = fma(xq[tt] - mq, xr[tt] - mr, acc);
+        for (int u = 0; u < W; ++u) {
+            delta[u] = delta0 + (long long)a * CW + c * W + u;
+            lo[u] = max(r0, max(0ll, -delta[u]));
+            hi[u] = min(r1, n - max(delta[u], 0ll));
+            if (delta[u] > p.delta_hi) hi[u] = lo[u];
+        }
+        int dlt[W], lo32[W], hi32[W];  // positions and diagonals fit in 32 bits (n < 2^31)
+#pragma unroll
+        for (int u = 0; u < W; ++u) { dlt[u] = (int)delta[u]; lo32[u] = (int)lo[u]; hi32[u] = (int)hi[u]; }
+
+        // seeds: direct centred dot products at row lo (reading G8),
+        // compensated (Kahan) accumulation.  Operands are position-major and padded to D
+        // dims, so a lane (G == 1) loads its DL dims of a window position as vectors.
+        T QT[W][DL];
+#pragma unroll
+        for (int u = 0; u < W; ++u) {
+            const bool ok = lo[u] < hi[u];
+            T mq[DL], mr[DL], cmp[DL];
+            const long long i0 = ok ? lo[u] : 0, j0 = ok ? lo[u] + delta[u] : 0;
+            load_dims<T, DL, G>(mu_q + i0 * D, g, mq);
+            load_dims<T, DL, G>(mu_r + j0 * D, g, mr);
+#pragma unroll
+            for (int kk = 0; kk < DL; ++kk) {
+                QT[u][kk] = (kk * G + g) >= d ? (T)-1 : (T)0;
+                cmp[kk] = (T)0;
             }
-            QT[kk] = acc;
+            if (ok) {
+                const T* xq_p = tw_q + i0 * D;
+                const T* xr_p = tw_r + j0 * D;
+#pragma unroll 2
+                for (int tt = 0; tt < m; ++tt) {
+                    T xq[DL], xr[DL];
+                    load_dims<T, DL, G>(xq_p + (long long)tt * D, g, xq);
+                    load_dims<T, DL, G>(xr_p + (long long)tt * D, g, xr);
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) {
+                        const T y = (xq[kk] - mq[kk]) * (xr[kk] - mr[kk]) - cmp[kk];
+                        const T t2 = QT[u][kk] + y;
+                        cmp[kk] = (t2 - QT[u][kk]) - y;
+                        QT[u][kk] = t2;
+                    }
+                }
+#pragma unroll
+                for (int kk = 0; kk < DL; ++kk)
+                    if ((kk * G + g) >= d) QT[u][kk] = (T)-1;  // padded dims (zero data)
+            }
         }
 
-        const int s_end = (int)(r1 - r0) + CA * (RA - 1);
-        const long long c0 = r0 + delta0;  // column of cell c = 0 at step 0
-        for (int cc = 0; cc < CA - 1; ++cc) enter(false, c0 + cc, st_r);
+        const int nrows = (int)(r1 - r0);
+        const int s_end = nrows + CW * (RA - 1);
+        const int R0 = (int)r0, C0 = (int)(r0 + delta0);  // row / column of step 0, cell 0
+        // batch pipeline bookkeeping (positions relative to R0 / C0)
+        int row_in = min(SB, nrows), col_in = min(SB, s_end) + CW - 1, row_out = 0, col_out = 0;
+        stage(true, R0, 0, row_in);
+        stage(false, C0, 0, col_in);
+        cp_async_commit();
+        cp_async_wait_all();
+        __syncwarp();
 
-        for (int s = 0; s < s_end; ++s) {
-            __syncwarp();
-            if (s >= 1) leave(false, c0 + s - 1);
-            if (s - 1 - CA * (RA - 1) >= 0) leave(true, r0 + s - 1 - CA * (RA - 1));
-            if (s < r1 - r0) enter(true, r0 + s, st_q);
-            enter(false, c0 + s + CA - 1, st_r);
-            __syncwarp();
+        // W == 2: column data of cell u = 0 is carried from cell u = 1 of the previous step
+        constexpr int CD = W == 2 ? DL : 1;
+        V4 carA[CD], carB[CD];
+        if constexpr (W == 2) {
+            const int sc0 = Gm::scol(C0 + c * W);
+#pragma unroll
+            for (int kk = 0; kk < DL; ++kk) carA[kk] = colv[kk * PSC + sc0];
+        }
 
-            const long long row = r0 + s - CA * a;
-            const long long col = row + delta;
-            const bool active = row >= lo && row < hi;
-            const bool upd = row > lo && row < hi;
-            const int sr = Gm::srow(row), sc = Gm::scol(col);
+        // one step: cells (row, row + delta[u]) of this lane
+        auto step = [&](int s, V4 (&Cold)[CD], V4 (&Cnew)[CD]) {
+            const int row = R0 + s - CW * a;
+            const int sr = Gm::srow(row);
+            bool active[W], upd[W];
+            int col[W];
+#pragma unroll
+            for (int u = 0; u < W; ++u) {
+                col[u] = row + dlt[u];
+                active[u] = row >= lo32[u] && row < hi32[u];
+                upd[u] = row > lo32[u] && row < hi32[u];
+            }
+            const int scn = Gm::scol(col[W - 1]);
 
             // thresholds stay in registers for small per-lane dim counts; wide lanes
             // re-read them from the ring after the sort (register budget)
-            constexpr bool KEEP = (DL <= 16 && G == 1);
-            T S[DL], tr[KEEP ? DL : 1], tc[KEEP ? DL : 1];
+            constexpr bool KEEP = (DL <= 16);
+            T S[W][DL], tr[KEEP ? DL : 1], tc0[KEEP ? DL : 1];
 #pragma unroll
             for (int kk = 0; kk < DL; ++kk) {
                 const int pl = kk * G + g;
                 const V4 R = rowv[pl * PSR + sr];
-                const V4 C = colv[pl * PSC + sc];
-                if (upd) QT[kk] = fma(R.x, C.y, fma(C.x, R.y, QT[kk]));   // Eq. (1) recurrence
-                const T aa = R.z * C.z;
-                S[kk] = PT<T>::sqrt_abs(fma(-QT[kk], aa, two_m));            // Eq. (1) distance
+                const V4 C = colv[pl * PSC + scn];
+                if constexpr (W == 2) {
+                    const V4 C0v = Cold[kk];
+                    if (upd[0]) QT[0][kk] = fma(R.x, C0v.y, fma(C0v.x, R.y, QT[0][kk]));   // Eq. (1)
+                    S[0][kk] = PT<T>::sqrt_abs(fma(-QT[0][kk], R.z * C0v.z, two_m));
+                    if constexpr (KEEP) tc0[kk] = C0v.w;
+                    Cnew[kk] = C;
+                }
+                if (upd[W - 1]) QT[W - 1][kk] = fma(R.x, C.y, fma(C.x, R.y, QT[W - 1][kk]));
+                S[W - 1][kk] = PT<T>::sqrt_abs(fma(-QT[W - 1][kk], R.z * C.z, two_m));  // Eq. (1)
                 if constexpr (KEEP) {
                     tr[kk] = R.w;
-                    tc[kk] = C.w;
+                    if constexpr (W == 1) tc0[kk] = C.w;
                 }
             }
-            sort_net<T, DL>(S);                                              // Eq. (2) sort
-            if (G > 1) lane_merge<T, DL, G>(S, g);
 #pragma unroll
-            for (int kk = 1; kk < DL; ++kk) S[kk] += S[kk - 1];              // Eq. (2) scan
-            if (G > 1) {
-                T tot = S[DL - 1];
+            for (int u = 0; u < W; ++u) {
+                sort_net<T, DL>(S[u]);                                               // Eq. (2) sort
+                if (G > 1) lane_merge<T, DL, G>(S[u], g);
+                // Eq. (2) inclusive scan, two independent half chains joined at the end
+                // (shorter dependency chain; summation order differs only by rounding)
+                if constexpr (DL >= 8) {
 #pragma unroll
-                for (int dd = 1; dd < G; dd <<= 1) {
-                    T y = __shfl_up_sync(FULL, tot, dd, G);
-                    if (g >= dd) tot += y;
+                    for (int kk = 1; kk < DL / 2; ++kk) S[u][kk] += S[u][kk - 1];
+#pragma unroll
+                    for (int kk = DL / 2 + 1; kk < DL; ++kk) S[u][kk] += S[u][kk - 1];
+#pragma unroll
+                    for (int kk = DL / 2; kk < DL; ++kk) S[u][kk] += S[u][DL / 2 - 1];
+                } else {
+#pragma unroll
+                    for (int kk = 1; kk < DL; ++kk) S[u][kk] += S[u][kk - 1];
                 }
-                T excl = __shfl_up_sync(FULL, tot, 1, G);
-                if (g == 0) excl = (T)0;
+                if (G > 1) {
+                    T tot = S[u][DL - 1];
 #pragma unroll
-                for (int kk = 0; kk < DL; ++kk) S[kk] += excl;
+                    for (int dd = 1; dd < G; dd <<= 1) {
+                        T y = __shfl_up_sync(FULL, tot, dd, G);
+                        if (g >= dd) tot += y;
+                    }
+                    T excl = __shfl_up_sync(FULL, tot, 1, G);
+                    if (g == 0) excl = (T)0;
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) S[u][kk] += excl;
+                }
             }
             bool hit = false;
 #pragma unroll
-            for (int kk = 0; kk < DL; ++kk) {
-                const int pl = kk * G + g;
-                if constexpr (KEEP) {
-                    hit |= S[kk] <= tr[kk];
-                    if (SELF) hit |= S[kk] <= tc[kk];
-                } else {
-                    hit |= S[kk] <= rowv[pl * PSR + sr].w;
-                    if (SELF) hit |= S[kk] <= colv[pl * PSC + sc].w;
+            for (int u = 0; u < W; ++u) {
+                bool h[4] = {false, false, false, false};  // independent predicate chains (ILP)
+#pragma unroll
+                for (int kk = 0; kk < DL; ++kk) {
+                    if constexpr (KEEP) {
+                        h[kk & 3] |= S[u][kk] <= tr[kk];
+                        if (SELF) {
+                            if constexpr (W == 2) h[kk & 3] |= S[u][kk] <= (u == 0 ? tc0[kk] : Cnew[kk].w);
+                            else h[kk & 3] |= S[u][kk] <= tc0[kk];
+                        }
+                    } else {
+                        const int pl = kk * G + g;
+                        h[kk & 3] |= S[u][kk] <= rowv[pl * PSR + sr].w;
+                        if (SELF) h[kk & 3] |= S[u][kk] <= colv[pl * PSC + Gm::scol(col[u])].w;
+                    }
                 }
+                hit |= ((h[0] | h[1]) | (h[2] | h[3])) && active[u];
             }
-            hit = hit && active;
             if (__any_sync(FULL, hit)) {
                 // Eq. (3) with the lowest-index tie rule: group min by shuffles, one leader
                 // per row / column group compares (value, index) with the ring's best.
 #pragma unroll
-                for (int kk = 0; kk < DL; ++kk) ssc[kk * 32 + lane] = active ? S[kk] : INF;
+                for (int u = 0; u < W; ++u)
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) ssc[(u * DL + kk) * 32 + lane] = active[u] ? S[u][kk] : INF;
                 __syncwarp();
 #pragma unroll 1
                 for (int kk = 0; kk < DL; ++kk) {
                     const int pl = kk * G + g;
-                    const T v = ssc[kk * 32 + lane];
-                    T vr = v;
+                    T v[W];
+#pragma unroll
+                    for (int u = 0; u < W; ++u) v[u] = ssc[(u * DL + kk) * 32 + lane];
+                    // row group: W cells per lane x CA lanes
+                    T vr = v[0];
+#pragma unroll
+                    for (int u = 1; u < W; ++u) vr = PT<T>::vmin(vr, v[u]);
 #pragma unroll
                     for (int bit = 0; bit < Gm::LOG_CA; ++bit)
                         vr = PT<T>::vmin(vr, __shfl_xor_sync(FULL, vr, 1 << (bit + Gm::LOG_G)));
-                    const unsigned eqr = __ballot_sync(FULL, v == vr) & gmask_row;
+                    bool mine = false;
+#pragma unroll
+                    for (int u = 0; u < W; ++u) mine |= v[u] == vr;
+                    const unsigned eqr = __ballot_sync(FULL, mine) & gmask_row;
                     if (vr < INF && lane == __ffs(eqr) - 1) {
+                        int j = col[W - 1];
+#pragma unroll
+                        for (int u = W - 1; u >= 0; --u)
+                            if (v[u] == vr) j = col[u];                 // lowest column first
                         const int ix = pl * PSR + sr;
                         const T cur = rowv[ix].w;
                         const unsigned ci = rowi[ix] & ~DIRTY;
-                        if (vr < cur || (vr == cur && (unsigned)col < ci)) {
+                        if (vr < cur || (vr == cur && (unsigned)j < ci)) {
                             rowv[ix].w = vr;
-                            rowi[ix] = (unsigned)col | DIRTY;
+                            rowi[ix] = (unsigned)j | DIRTY;
+                            rowdirty[sr] = 1;
                         }
                     }
                     if (SELF) {
-                        T vc = v;
 #pragma unroll
-                        for (int bit = 0; bit < 5 - Gm::LOG_G - Gm::LOG_CA; ++bit)
-                            vc = PT<T>::vmin(vc, __shfl_xor_sync(FULL, vc, 1 << (bit + Gm::LOG_G + Gm::LOG_CA)));
-                        const unsigned eqc = __ballot_sync(FULL, v == vc) & gmask_col;
-                        // lowest row index = highest a = highest lane
-                        if (vc < INF && eqc != 0 && lane == 31 - __clz(eqc)) {
-                            const int ix = pl * PSC + sc;
-                            const T cur = colv[ix].w;
-                            const unsigned ci = coli[ix] & ~DIRTY;
-                            if (vc < cur || (vc == cur && (unsigned)row < ci)) {
-                                colv[ix].w = vc;
-                                coli[ix] = (unsigned)row | DIRTY;
+                        for (int u = 0; u < W; ++u) {
+                            T vc = v[u];
+#pragma unroll
+                            for (int bit = 0; bit < 5 - Gm::LOG_G - Gm::LOG_CA; ++bit)
+                                vc = PT<T>::vmin(vc, __shfl_xor_sync(FULL, vc, 1 << (bit + Gm::LOG_G + Gm::LOG_CA)));
+                            const unsigned eqc = __ballot_sync(FULL, v[u] == vc) & gmask_col;
+                            // lowest row index = highest a = highest lane
+                            if (vc < INF && eqc != 0 && lane == 31 - __clz(eqc)) {
+                                const int scu = Gm::scol(col[u]);
+                                const int ix = pl * PSC + scu;
+                                const T cur = colv[ix].w;
+                                const unsigned ci = coli[ix] & ~DIRTY;
+                                if (vc < cur || (vc == cur && (unsigned)row < ci)) {
+                                    colv[ix].w = vc;
+                                    coli[ix] = (unsigned)row | DIRTY;
+                                    coldirty[scu] = 1;
+                                }
                             }
                         }
                     }
                 }
+                __syncwarp();
             }
+        };
+
+        for (int s0 = 0; s0 < s_end; s0 += SB) {
+            // evict positions no step from s0 on reads; prefetch the next batch's entries
+            const int rx = min(max(s0 - CW * (RA - 1), 0), nrows);
+            evict(true, R0, row_out, rx);
+            row_out = rx;
+            evict(false, C0, col_out, s0);
+            col_out = s0;
+            const int nxt = min(s0 + 2 * SB, s_end);
+            const int r_need = min(nxt, nrows), c_need = nxt + CW - 1;
+            stage(true, R0, row_in, r_need);
+            stage(false, C0, col_in, c_need);
+            row_in = max(row_in, r_need);
+            col_in = max(col_in, c_need);
+            cp_async_commit();
+#pragma unroll
+            for (int k2 = 0; k2 < SB; k2 += 2) {
+                if (s0 + k2 < s_end) step(s0 + k2, carA, carB);
+                if (s0 + k2 + 1 < s_end) step(s0 + k2 + 1, carB, carA);
+            }
+            cp_async_wait_all();   // this lane's prefetch for the next batch has landed
+            __syncwarp();          // ... and everyone's; all reads of this batch are done
         }
-        __syncwarp();
-        // epilogue: the last row and the last CA columns are still in the rings
-        if (r1 - r0 >= 1) leave(true, r1 - 1);
-        for (int v = s_end - 1; v <= s_end + CA - 2; ++v) leave(false, c0 + v);
+        // epilogue: evict what is still in the rings
+        evict(true, R0, row_out, nrows);
+        evict(false, C0, col_out, col_in);
         __syncwarp();
     }
 }
 
-
-template <class T, int DL, int G, bool SELF> struct Inst {
+template <class T, int DL, int G, int W, bool SELF> struct Inst {
     static size_t smem();
     static cudaError_t launch(const MainParams& p, int grid, cudaStream_t s);
     static int blocks_per_sm();
+    static int warps_per_block() { return Smem<T, DL, G, W>::WPB; }
 };
 
 #ifdef MP_DIAG_IMPL
-template <class T, int DL, int G, bool SELF> size_t Inst<T, DL, G, SELF>::smem() {
-    return Smem<T, DL, G>::bytes_per_warp * WARPS_PER_BLOCK;
+template <class T, int DL, int G, int W, bool SELF> size_t Inst<T, DL, G, W, SELF>::smem() {
+    return Smem<T, DL, G, W>::bytes_per_warp * Smem<T, DL, G, W>::WPB;
 }
-template <class T, int DL, int G, bool SELF>
-cudaError_t Inst<T, DL, G, SELF>::launch(const MainParams& p, int grid, cudaStream_t s) {
+template <class T, int DL, int G, int W, bool SELF>
+cudaError_t Inst<T, DL, G, W, SELF>::launch(const MainParams& p, int grid, cudaStream_t s) {
     const size_t sm = smem();
-    cudaError_t e = cudaFuncSetAttribute(mp_diag<T, DL, G, SELF>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaError_t e = cudaFuncSetAttribute(mp_diag<T, DL, G, W, SELF>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
-    mp_diag<T, DL, G, SELF><<<grid, WARPS_PER_BLOCK * 32, sm, s>>>(p);
+    mp_diag<T, DL, G, W, SELF><<<grid, Smem<T, DL, G, W>::WPB * 32, sm, s>>>(p);
     return cudaGetLastError();
 }
-template <class T, int DL, int G, bool SELF> int Inst<T, DL, G, SELF>::blocks_per_sm() {
+template <class T, int DL, int G, int W, bool SELF> int Inst<T, DL, G, W, SELF>::blocks_per_sm() {
     const size_t sm = smem();
-    cudaFuncSetAttribute(mp_diag<T, DL, G, SELF>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaFuncSetAttribute(mp_diag<T, DL, G, W, SELF>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     int nb = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mp_diag<T, DL, G, SELF>, WARPS_PER_BLOCK * 32, sm);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mp_diag<T, DL, G, W, SELF>, Smem<T, DL, G, W>::WPB * 32, sm);
     return nb;
 }
 #endif
-
-
 
 }  // namespace mpk

@@ -10,9 +10,9 @@ namespace mpk {
 struct MainParams {
     const void* st_q;   // stats, position-major [pos][dim], V4 = (df, dg, a, 0)   (query / rows)
     const void* st_r;   // stats of the reference series (columns); == st_q for self-join
-    const void* tw_q;   // working-precision series [dim][t], t < L (seeds)
+    const void* tw_q;   // working-precision series, position-major padded [t][Dp], t < L (seeds)
     const void* tw_r;
-    const void* mu_q;   // working-precision window means [dim][pos]
+    const void* mu_q;   // working-precision window means, position-major padded [pos][Dp]
     const void* mu_r;
     void* keys;         // merge keys [pos][rank] of the QUERY profile (self-join: the one profile)
     const long long* seg_prefix;  // exclusive prefix of #segments per diagonal block (NB+1)
@@ -27,8 +27,10 @@ struct MainParams {
 struct PreParams {
     const double* T;    // input [dim][t] FP64, L = n + m - 1
     void* st;           // out stats [pos][dim]
-    void* tw;           // out working series [dim][t] (may alias nothing; FP64 mode: unused)
+    void* tw;           // out working series, position-major padded [t][Dp], t < L (seeds)
     void* mu;           // out window mean [dim][pos]
+    void* mup;          // out window mean, position-major padded [pos][Dp] (seeds)
+    int Dp;             // padded dimension count of the kernel variant (DL * G)
     float* nrm32;       // scratch for FP32 path (norm) [dim][pos]
     double* nrm64;
     long long n;
@@ -39,10 +41,10 @@ struct PreParams {
 enum { P64 = 0, P32 = 1, P16 = 2, PMIX = 3 };
 
 // Variant selection for a given (precision, d): dims per lane DL and lanes per cell G.
-struct Variant { int DL; int G; int NC; };
+struct Variant { int DL; int G; int W; int NC; };
 Variant pick_variant(int prec, int d);
 size_t smem_per_block(int prec, int d, bool self);
-int warps_per_block();
+int variant_warps_per_block(int prec, int d, bool self);
 
 // Launchers (return cudaError_t).
 cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s);

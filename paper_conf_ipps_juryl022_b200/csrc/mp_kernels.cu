@@ -18,13 +18,24 @@ __global__ void pre_stats(const PreParams p) {
     const int dim = (int)(gid / n);
     const long long pos = gid % n;
     const double* x = p.T + (long long)dim * L + pos;
-    T s = 0;
-    for (int t = 0; t < m; ++t) s += (T)x[t];
+    // two-pass with compensated (Kahan) sums in the precalc precision; the paper leaves the
+    // precalculation formulas out and stresses its accuracy (L792-794)
+    T s = 0, c = 0;
+    for (int t = 0; t < m; ++t) {
+        const T y = (T)x[t] - c;
+        const T tt = s + y;
+        c = (tt - s) - y;
+        s = tt;
+    }
     const T mu = s / (T)m;
     T q = 0;
+    c = 0;
     for (int t = 0; t < m; ++t) {
         const T cx = (T)x[t] - mu;
-        q = fma(cx, cx, q);
+        const T y = cx * cx - c;
+        const T tt = q + y;
+        c = (tt - q) - y;
+        q = tt;
     }
     reinterpret_cast<T*>(p.mu)[(long long)dim * n + pos] = mu;
     const T nr = sqrt(q);
@@ -58,9 +69,20 @@ __global__ void pre_diff(const PreParams p) {
     reinterpret_cast<V4*>(p.st)[pos * d + dim] = v;
 }
 
-__global__ void to_f32(const double* x, float* y, long long count) {
-    const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-    if (i < count) y[i] = (float)x[i];
+// position-major, zero-padded copies of the working-precision series and window means
+// (the seeds' operands: a lane's dims are contiguous, so they load as vectors)
+template <class T>
+__global__ void pre_pm(const PreParams p) {
+    const long long n = p.n, L = p.n + p.m - 1;
+    const int d = p.d, Dp = p.Dp;
+    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (gid >= L * Dp) return;
+    const long long t = gid / Dp;
+    const int dim = (int)(gid % Dp);
+    T* tw = reinterpret_cast<T*>(p.tw);
+    T* mup = reinterpret_cast<T*>(p.mup);
+    tw[gid] = dim < d ? (T)p.T[(long long)dim * L + t] : (T)0;
+    if (t < n) mup[gid] = dim < d ? reinterpret_cast<const T*>(p.mu)[(long long)dim * n + t] : (T)0;
 }
 
 // ------------------------------------------------------------------ keys
@@ -77,12 +99,12 @@ __global__ void keys64_to_ext(const K64* k, long long* ext, long long count) {
     const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
     if (i < count) {
         ext[i] = (long long)k[i].v;
-        ext[count + i] = (k[i].v == EMPTY64V) ? (long long)EMPTY64I : (long long)k[i].i;
+        ext[count + i] = (k[i].v == EMPTY64V) ? EXT_EMPTY : (long long)k[i].i;
     }
 }
 __global__ void key_mask(long long count, long long* ext, const long long* gv) {
     const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-    if (i < count && ext[i] != gv[i]) ext[count + i] = (long long)EMPTY64I;
+    if (i < count && ext[i] != gv[i]) ext[count + i] = EXT_EMPTY;
 }
 // ext keys [pos][rank] -> P [rank][pos] (sum / (k+1), reading G11), I [rank][pos]
 __global__ void finalize32(const unsigned long long* k, long long n, int d, double* P, long long* I) {
@@ -108,7 +130,7 @@ __global__ void finalize64(const long long* ext, long long n, int d, double* P, 
     const long long ix = ext[count + gid];
     double pv;
     long long oi;
-    if (v >= EMPTY64V || ix == (long long)EMPTY64I) { pv = __longlong_as_double(0x7ff0000000000000ll); oi = -1; }
+    if (v >= EMPTY64V || ix == EXT_EMPTY) { pv = __longlong_as_double(0x7ff0000000000000ll); oi = -1; }
     else { pv = __longlong_as_double((long long)v) / (double)(rk + 1); oi = ix; }
     P[(long long)rk * n + pos] = pv;
     I[(long long)rk * n + pos] = oi;
@@ -123,42 +145,53 @@ __global__ void check_finite(const double* x, long long count, int* flag) {
 static inline unsigned grid1d(long long count, int bs) { return (unsigned)((count + bs - 1) / bs); }
 
 Variant pick_variant(int prec, int d) {
-    // FP32: a lane holds up to 32 dims; FP64: up to 16 (register budget).
-    const int maxdl = prec == P64 ? 16 : 32;
+    // A lane holds DL <= 16 dims (register budget; DL = 32 only for FP32 d > 512); for small
+    // d a lane owns W = 2 adjacent diagonals (d <= 8).
     int dp = 1;
     while (dp < d) dp <<= 1;
     Variant v;
-    if (dp <= maxdl) { v.DL = dp; v.G = 1; }
-    else { v.DL = maxdl; v.G = dp / maxdl; }
-    v.NC = 32 / v.G;
+    if (prec == P64) {
+        if (dp <= 16) { v.DL = dp; v.G = 1; v.W = dp <= 8 ? 2 : 1; }
+        else { v.DL = 16; v.G = dp / 16; v.W = 1; }
+    } else {
+        if (dp <= 8) { v.DL = dp; v.G = 1; v.W = 2; }
+        else if (dp == 16) { v.DL = 16; v.G = 1; v.W = 1; }
+        else if (dp <= 512) { v.DL = 16; v.G = dp / 16; v.W = 1; }
+        else { v.DL = 32; v.G = dp / 32; v.W = 1; }
+    }
+    v.NC = 32 / v.G * v.W;
     return v;
 }
 
-int warps_per_block() { return WARPS_PER_BLOCK; }
-
-// op: 0 = smem, 1 = launch, 2 = blocks/SM
+// op: 0 = smem, 1 = launch, 2 = blocks/SM, 3 = warps/block
 template <class T, bool SELF>
-static long long dispatch_t(int op, int DL, int G, const MainParams* p, int grid, cudaStream_t s) {
-#define MP_CASE(dl, g)                                                                 \
-    if (DL == dl && G == g) {                                                          \
-        if (op == 0) return (long long)Inst<T, dl, g, SELF>::smem();                   \
-        if (op == 1) return (long long)Inst<T, dl, g, SELF>::launch(*p, grid, s);      \
-        return Inst<T, dl, g, SELF>::blocks_per_sm();                                  \
+static long long dispatch_t(int op, int DL, int G, int W, const MainParams* p, int grid, cudaStream_t s) {
+#define MP_CASE(dl, g, w)                                                                  \
+    if (DL == dl && G == g && W == w) {                                                    \
+        if (op == 0) return (long long)Inst<T, dl, g, w, SELF>::smem();                    \
+        if (op == 1) return (long long)Inst<T, dl, g, w, SELF>::launch(*p, grid, s);       \
+        if (op == 3) return Inst<T, dl, g, w, SELF>::warps_per_block();                    \
+        return Inst<T, dl, g, w, SELF>::blocks_per_sm();                                   \
     }
-    MP_CASE(1, 1) MP_CASE(2, 1) MP_CASE(4, 1) MP_CASE(8, 1) MP_CASE(16, 1)
-    if constexpr (sizeof(T) == 4) { MP_CASE(32, 1) MP_CASE(32, 2) MP_CASE(32, 4) MP_CASE(32, 8) MP_CASE(32, 16) MP_CASE(32, 32) }
-    else { MP_CASE(16, 2) MP_CASE(16, 4) MP_CASE(16, 8) MP_CASE(16, 16) MP_CASE(16, 32) }
+    if constexpr (sizeof(T) == 4) {
+        MP_CASE(1, 1, 2) MP_CASE(2, 1, 2) MP_CASE(4, 1, 2) MP_CASE(8, 1, 2) MP_CASE(16, 1, 1)
+        MP_CASE(16, 2, 1) MP_CASE(16, 4, 1) MP_CASE(16, 8, 1) MP_CASE(16, 16, 1) MP_CASE(16, 32, 1) MP_CASE(32, 32, 1)
+    } else {
+        MP_CASE(1, 1, 2) MP_CASE(2, 1, 2) MP_CASE(4, 1, 2) MP_CASE(8, 1, 2) MP_CASE(16, 1, 1)
+        MP_CASE(16, 2, 1) MP_CASE(16, 4, 1) MP_CASE(16, 8, 1) MP_CASE(16, 16, 1) MP_CASE(16, 32, 1)
+    }
 #undef MP_CASE
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
 }
 
 static long long dispatch(int op, int prec, bool self, int d, const MainParams* p, int grid, cudaStream_t s) {
     const Variant v = pick_variant(prec, d);
-    if (prec == P64) return self ? dispatch_t<double, true>(op, v.DL, v.G, p, grid, s) : dispatch_t<double, false>(op, v.DL, v.G, p, grid, s);
-    if (prec == P32) return self ? dispatch_t<float, true>(op, v.DL, v.G, p, grid, s) : dispatch_t<float, false>(op, v.DL, v.G, p, grid, s);
+    if (prec == P64) return self ? dispatch_t<double, true>(op, v.DL, v.G, v.W, p, grid, s) : dispatch_t<double, false>(op, v.DL, v.G, v.W, p, grid, s);
+    if (prec == P32) return self ? dispatch_t<float, true>(op, v.DL, v.G, v.W, p, grid, s) : dispatch_t<float, false>(op, v.DL, v.G, v.W, p, grid, s);
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
 }
 
+int variant_warps_per_block(int prec, int d, bool self) { return (int)dispatch(3, prec, self, d, nullptr, 0, 0); }
 size_t smem_per_block(int prec, int d, bool self) { return (size_t)dispatch(0, prec, self, d, nullptr, 0, 0); }
 int main_blocks_per_sm(int prec, int d, bool self) { return (int)dispatch(2, prec, self, d, nullptr, 0, 0); }
 cudaError_t launch_main(int prec, bool self, const MainParams& p, int grid, cudaStream_t s) {
@@ -171,10 +204,11 @@ cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s) {
     if (prec == P64) {
         pre_stats<double><<<grid1d(cnt, 256), 256, 0, s>>>(p);
         pre_diff<double><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+        pre_pm<double><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
     } else if (prec == P32) {
         pre_stats<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
         pre_diff<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-        to_f32<<<grid1d(L * p.d, 256), 256, 0, s>>>(p.T, reinterpret_cast<float*>(p.tw), L * p.d);
+        pre_pm<float><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
     } else {
         return cudaErrorInvalidValue;
     }

@@ -54,8 +54,7 @@ def test_band_plan(lib, cfg, world):
     assert bb[0] == 0 and np.all(np.diff(bb) >= 0)
     total = (n - e - 1) * (n - e) // 2 if self_join else n * n
     assert cells.sum() == total
-    nc = 32 // max(1, (1 << int(np.ceil(np.log2(d)))) // 32)
-    block_max = nc * n
+    block_max = 64 * n   # a diagonal block holds at most 64 diagonals
     assert cells.max() - cells.min() <= 2 * block_max
 
 
