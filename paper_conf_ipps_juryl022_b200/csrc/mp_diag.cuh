@@ -316,7 +316,6 @@ mp_diag(const MainParams p) {
 
     const long long n = p.n;
     const int d = p.d, m = p.m, H = p.H;
-    const long long L = n + m - 1;
     const T two_m = (T)(2 * m);
     const T INF = PT<T>::inf(), NINF = PT<T>::ninf();
 
@@ -344,6 +343,26 @@ mp_diag(const MainParams p) {
         const int ps = is_row ? PSR : PSC;
         const V4* __restrict__ st = is_row ? st_q : st_r;
         const bool want_thr = is_row || SELF;
+        if (d == D && base + p_lo >= 0 && base + p_hi <= n32 && want_thr) {
+            // common case: all positions in range, no padded dims -- branch-free copies
+            for (int e = lane; e < cnt * D; e += 32) {
+                const int pi = e / D, pl = e - pi * D;
+                const int pos = base + p_lo + pi;
+                const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
+                if (pl == 0) dflag[sl] = 0;
+                V4* dst = &buf[pl * ps + sl];
+                const V4* src = st + (size_t)pos * d + pl;
+                if constexpr (sizeof(T) == 4) {
+                    cp_async8(dst, src);
+                    cp_async4(&dst->z, &src->z);
+                } else {
+                    cp_async16(dst, src);
+                    cp_async8(&dst->z, &src->z);
+                }
+                KO::stage(keys + (size_t)pos * d + rank_of_plane<DL, G>(pl), &dst->w, &ib[pl * ps + sl]);
+            }
+            return;
+        }
         for (int e = lane; e < cnt * D; e += 32) {
             const int pi = e / D, pl = e - pi * D;
             const int pos = base + p_lo + pi;
