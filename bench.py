@@ -130,6 +130,14 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
+def load_traffic(config, prec):
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            return json.load(f).get(f"{config}/{prec}", {}).get("traffic_bytes")
+    except (OSError, ValueError):
+        return None
+
+
 def load_peaks():
     try:
         with open(PEAKS_PATH) as f:
@@ -139,15 +147,15 @@ def load_peaks():
 
 
 def launches_per_step(prec: str, self_join: bool) -> int:
-    # check_finite (1 per series) + precompute (pre_stats, pre_diff [+ to_f32]) per series
+    # check_finite (1 per series) + precompute (pre_stats, pre_diff, pre_pm) per series
     # + init_keys + mp_diag + [keys64_to_ext] + finalize
     series = 1 if self_join else 2
-    pre = 2 if prec == "fp64" else 3
+    pre = 3
     return series * (1 + pre) + 1 + 1 + (1 if prec == "fp64" else 0) + 1
 
 
 # ---------------------------------------------------------------------------- CPU oracle leg
-def oracle_sample(cfg, target_s: float = 15.0, max_rows: int = 4096):
+def oracle_sample(cfg, target_s: float = 15.0, max_rows: int = 8192):
     """Time the FP64 oracle (as it stands) on sampled query rows of the workload.
     Returns (cell*dims per second, rows, seconds, threads)."""
     import oracle
@@ -321,7 +329,8 @@ def main():
         peak_tops = SM_COUNT * ALU_LANES * NOMINAL_SM_MHZ * 1e6 / 1e12
         achieved = ops / (kms * 1e-3) / 1e12 if kms > 0 else None
         roof = {"bound": "alu", "achieved": achieved, "peak": peak_tops, "unit": "Tops/s",
-                "frac": achieved / peak_tops if achieved else None, "traffic": None,
+                "frac": achieved / peak_tops if achieved else None,
+                "traffic": load_traffic(args.config, args.precision),
                 "kernel": "mp_diag", "ops_per_cell_dim": alu_ops_per_cell_dim(d, self_join),
                 "computed_cell_dims": cells * d,
                 "peak_basis": f"148 SM x 64 ALU lanes/clk x {NOMINAL_SM_MHZ:.0f} MHz (derived; MEASURED_PEAKS {src} "

@@ -129,6 +129,12 @@ mp_status mp_finalize_device(mp_ctx* ctx, void* cuda_stream, int64_t d, int64_t 
 mp_status mp_plan_bands(int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
                         int self_join, int world, int64_t* block_begin, int64_t* cells);
 
+/* Diagonal range of each band: band g covers diagonals delta = j - i in
+ * [diag_begin[g], diag_begin[g+1]) (world+1 entries; self-join delta > exclusion, AB-join
+ * delta in (-n, n)).  Host only, no GPU needed. */
+mp_status mp_plan_diagonals(int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
+                            int self_join, int world, int64_t* diag_begin);
+
 /* Kernel timing of the last mp_compute* / mp_partial_device call on ctx (ms, CUDA
  * events around the main diagonal kernel only) and its launch count. */
 mp_status mp_last_timing(const mp_ctx* ctx, double* main_kernel_ms, int64_t* launches);

@@ -307,6 +307,20 @@ mp_status mp_plan_bands(int64_t d, int64_t n, int64_t m, mp_precision prec, int6
     return MP_OK;
 }
 
+mp_status mp_plan_diagonals(int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
+                            int self_join, int world, int64_t* diag_begin) {
+    if (world < 1 || !diag_begin || d < 1 || n < 2 || m < 2 || prec < 0 || prec > 3) return MP_ERR_INVALID;
+    if (self_join && exclusion < 0) exclusion = (m + 3) / 4;
+    Plan pl = build_plan(d, n, exclusion, self_join != 0, prec, default_h(prec, m));
+    if (pl.nb == 0) {
+        for (int g = 0; g <= world; ++g) diag_begin[g] = pl.dlo;
+        return MP_OK;
+    }
+    std::vector<int64_t> bb = band_blocks(pl, world);
+    for (int g = 0; g <= world; ++g) diag_begin[g] = std::min<int64_t>(pl.dlo + bb[g] * pl.nc, pl.dhi + 1);
+    return MP_OK;
+}
+
 mp_status mp_partial_device(mp_ctx* ctx, void* cuda_stream, const double* dT, const double* dTr,
                             int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
                             int rank, int world, int64_t* dKeys) {

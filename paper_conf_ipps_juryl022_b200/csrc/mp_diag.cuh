@@ -238,13 +238,14 @@ constexpr int ilog2(int x) { int l = 0; while ((1 << l) < x) ++l; return l; }
 
 template <int G, int W> struct Geo {
     static constexpr int NL = 32 / G;                                   // lane-cells per warp
-    static constexpr int CA = NL >= 16 ? 4 : (NL >= 4 ? 2 : 1);         // lane-cells per row group
+    // lane-cells per row group: 8 x 4 (rows x lanes) for one cell per lane, else 4 columns
+    static constexpr int CA = (W == 1 && NL == 32) ? 8 : NL >= 16 ? 4 : (NL >= 4 ? 2 : 1);
     static constexpr int RA = NL / CA;                                   // distinct rows per step
     static constexpr int CW = CA * W;                                    // distinct columns per step
     static constexpr int NC = NL * W;                                    // cells (diagonals) per warp
     // ring positions move in batches of SB steps, prefetched one batch ahead: live rows
     // span CW(RA-1) + 2 SB, live columns 2 SB + CW - 1
-    static constexpr int SB = 2;
+    static constexpr int SB = W == 1 ? 4 : 2;
     static constexpr int RING_R = pow2ceil(CW * (RA - 1) + 2 * SB) < CW ? CW : pow2ceil(CW * (RA - 1) + 2 * SB);
     static constexpr int RPC = RING_R / CW;                              // ring rows per residue class
     static constexpr int RING_C = pow2ceil(2 * SB + CW - 1);
@@ -401,7 +402,7 @@ mp_diag(const MainParams p) {
         const int ps = is_row ? PSR : PSC;
         // early out: most evictions find nothing dirty
         bool any = false;
-        for (int pi = lane; pi < cnt; pi += 32) {
+        for (int pi = lane; pi < cnt; pi += 32) {  // one pass in steady state (cnt = SB)
             const int pos = base + p_lo + pi;
             if (pos >= 0 && pos < n32) any |= dflag[is_row ? Gm::srow(pos) : Gm::scol(pos)] != 0;
         }
@@ -676,10 +677,16 @@ mp_diag(const MainParams p) {
             row_in = max(row_in, r_need);
             col_in = max(col_in, c_need);
             cp_async_commit();
+            if constexpr (W == 2) {  // ping-pong the carried column registers (no moves)
 #pragma unroll
-            for (int k2 = 0; k2 < SB; k2 += 2) {
-                if (s0 + k2 < s_end) step(s0 + k2, carA, carB);
-                if (s0 + k2 + 1 < s_end) step(s0 + k2 + 1, carB, carA);
+                for (int k2 = 0; k2 < SB; k2 += 2) {
+                    if (s0 + k2 < s_end) step(s0 + k2, carA, carB);
+                    if (s0 + k2 + 1 < s_end) step(s0 + k2 + 1, carB, carA);
+                }
+            } else {  // one copy of the step body (instruction-cache footprint)
+                const int s1 = min(s0 + SB, s_end);
+#pragma unroll 1
+                for (int ss = s0; ss < s1; ++ss) step(ss, carA, carB);
             }
             cp_async_wait_all();   // this lane's prefetch for the next batch has landed
             __syncwarp();          // ... and everyone's; all reads of this batch are done

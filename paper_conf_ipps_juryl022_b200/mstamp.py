@@ -23,7 +23,7 @@ STATUS = {0: "MP_OK", 1: "MP_ERR_INVALID", 2: "MP_ERR_NOMEM", 3: "MP_ERR_CUDA", 
           5: "MP_ERR_UNSUPPORTED"}
 EXPORTS = ["mp_init", "mp_free", "mp_last_error", "mp_version", "mp_compute", "mp_compute_device",
            "mp_key_words", "mp_partial_device", "mp_key_mask_device", "mp_finalize_device",
-           "mp_plan_bands", "mp_last_timing"]
+           "mp_plan_bands", "mp_plan_diagonals", "mp_last_timing"]
 
 _lib = None
 
@@ -69,6 +69,8 @@ def load():
     lib.mp_finalize_device.restype = i32
     lib.mp_plan_bands.argtypes = [i64, i64, i64, i32, i64, i32, i32, p, p]
     lib.mp_plan_bands.restype = i32
+    lib.mp_plan_diagonals.argtypes = [i64, i64, i64, i32, i64, i32, i32, p]
+    lib.mp_plan_diagonals.restype = i32
     lib.mp_last_timing.argtypes = [p, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(i64)]
     lib.mp_last_timing.restype = i32
     _lib = lib
@@ -95,6 +97,17 @@ def plan_bands(d, n, m, prec="fp32", exclusion=-1, self_join=True, world=1):
     if st != 0:
         raise MPError(st, "mp_plan_bands")
     return bb, cells
+
+
+def plan_diagonals(d, n, m, prec="fp32", exclusion=-1, self_join=True, world=1):
+    """Host scheduler: band g covers diagonals [diag_begin[g], diag_begin[g+1])."""
+    lib = load()
+    db = np.zeros(world + 1, dtype=np.int64)
+    st = lib.mp_plan_diagonals(d, n, m, _prec(prec), exclusion, int(bool(self_join)), world,
+                               db.ctypes.data_as(ctypes.c_void_p))
+    if st != 0:
+        raise MPError(st, "mp_plan_diagonals")
+    return db
 
 
 def key_words(d, n, prec="fp32") -> int:
@@ -201,11 +214,12 @@ class Context:
         return ms.value, nl.value
 
 
-def merge_partials(ctx: Context, keys, d, n, prec, group=None):
+def merge_partials(ctx: Context, keys, d, n, prec, group=None, mask=None):
     """MINLOC all-reduce of partial keys over the process group (the path's one exchange).
 
     FP32/FP16/MIXED: one int64 MIN.  FP64: MIN on the value plane, mask indices whose
-    value lost, MIN on the index plane.  ``keys`` is modified in place.
+    value lost (mp_key_mask_device), MIN on the index plane.  ``keys`` is
+    modified in place.  ``mask`` overrides the mask step (CPU protocol tests only).
     """
     import torch.distributed as dist
     count = d * n
@@ -213,7 +227,10 @@ def merge_partials(ctx: Context, keys, d, n, prec, group=None):
         v = keys[:count]
         gv = v.clone()
         dist.all_reduce(gv, op=dist.ReduceOp.MIN, group=group)
-        ctx.key_mask_device(d, n, keys, gv)
+        if mask is None:
+            ctx.key_mask_device(d, n, keys, gv)
+        else:
+            mask(keys, gv)
         v.copy_(gv)
         dist.all_reduce(keys[count:], op=dist.ReduceOp.MIN, group=group)
     else:

@@ -16,7 +16,11 @@ Tr = None if cfg["Tr"] is None else torch.from_numpy(cfg["Tr"]).cuda()
 P = torch.empty(d, n, dtype=torch.float64, device="cuda")
 I = torch.empty(d, n, dtype=torch.int64, device="cuda")
 ctx = mstamp.Context(0)
+import subprocess  # noqa: E402
 for r in range(reps):
     ctx.compute_device(T, m, P, I, prec, e, Tr=Tr)
+    ctx.compute_device(T, m, P, I, prec, e, Tr=Tr)
+    clk = subprocess.run(["nvidia-smi", "--query-gpu=clocks.sm", "--format=csv,noheader,nounits"],
+                         capture_output=True, text=True).stdout.strip()
     torch.cuda.synchronize()
-    print(cfg["d"], n, prec, "main kernel ms", ctx.last_timing())
+    print(cfg["d"], n, prec, "main kernel ms", ctx.last_timing(), "sm_mhz(after)", clk)
