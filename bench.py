@@ -295,7 +295,7 @@ def main():
 
     per_prec = {}
     if not args.no_per_precision:
-        for prec in ("fp64", "fp32"):
+        for prec in ("fp64", "fp32", "mixed", "fp16"):
             if prec == args.precision:
                 per_prec[prec] = {"value": value, "ms_per_step": ms, "main_kernel_ms": kms}
                 continue

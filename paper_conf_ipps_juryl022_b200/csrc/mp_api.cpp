@@ -46,6 +46,7 @@ struct mp_ctx {
     std::string err;
     // cached scratch
     Buf dT, dTr, st_q, st_r, tw_q, tw_r, mu_q, mu_r, mup_q, mup_r, nrm, keys, ext, seg, counter, dP, dI, flag;
+    Buf stp_q, stp_r, scale, maxbits, flat;  // FP16 / Mixed precompute
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     double last_ms = 0.0;
     int64_t last_launches = 0;
@@ -142,7 +143,6 @@ mp_status validate(mp_ctx* ctx, const void* T, int64_t d, int64_t n, int64_t m, 
     if (n >= (int64_t(1) << 31) - 1) return fail(ctx, MP_ERR_INVALID, "n must be < 2^31");
     if (m > (int64_t(1) << 20)) return fail(ctx, MP_ERR_INVALID, "m too large");
     if (prec < 0 || prec > 3) return fail(ctx, MP_ERR_INVALID, "unknown precision");
-    if (prec == MP_FP16 || prec == MP_MIXED) return fail(ctx, MP_ERR_UNSUPPORTED, "FP16/MIXED not built yet");
     if (prec == MP_FP64 && d > 512) return fail(ctx, MP_ERR_UNSUPPORTED, "FP64 supports d <= 512");
     return MP_OK;
 }
@@ -167,28 +167,36 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     if (flag) return fail(ctx, MP_ERR_INVALID, "non-finite input");
 
     // precalculation (Pseudocode 1 line 2)
-    MP_CUDA(ctx, ensure(ctx->st_q, (size_t)n * d * 4 * eb));
+    const bool half = prec == MP_FP16 || prec == MP_MIXED;
+    const size_t sb = half ? 16 : 4 * eb;                                   // stats entry bytes
+    const size_t tb = prec == MP_FP64 ? 8 : (prec == MP_FP16 ? 2 : 4);       // precalc value bytes
     const mpk::Variant var = mpk::pick_variant(prec, (int)d);
     const int Dp = var.DL * var.G;
-    MP_CUDA(ctx, ensure(ctx->mu_q, (size_t)n * d * eb));
-    MP_CUDA(ctx, ensure(ctx->mup_q, (size_t)n * Dp * eb));
-    MP_CUDA(ctx, ensure(ctx->nrm, (size_t)n * d * eb));
-    MP_CUDA(ctx, ensure(ctx->tw_q, (size_t)L * Dp * eb));
     mpk::PreParams pp{};
     pp.n = n; pp.d = (int)d; pp.m = (int)m; pp.Dp = Dp;
+    MP_CUDA(ctx, ensure(ctx->nrm, (size_t)n * d * tb));
     pp.nrm32 = (float*)ctx->nrm.p; pp.nrm64 = (double*)ctx->nrm.p;
-    pp.T = dT; pp.st = ctx->st_q.p; pp.mu = ctx->mu_q.p; pp.tw = ctx->tw_q.p; pp.mup = ctx->mup_q.p;
-    MP_CUDA(ctx, mpk::launch_precompute(prec, pp, s));
-    if (!self) {
-        MP_CUDA(ctx, ensure(ctx->st_r, (size_t)n * d * 4 * eb));
-        MP_CUDA(ctx, ensure(ctx->mu_r, (size_t)n * d * eb));
-        MP_CUDA(ctx, ensure(ctx->mup_r, (size_t)n * Dp * eb));
-        MP_CUDA(ctx, ensure(ctx->tw_r, (size_t)L * Dp * eb));
-        pp.T = dTr; pp.st = ctx->st_r.p; pp.mu = ctx->mu_r.p; pp.tw = ctx->tw_r.p; pp.mup = ctx->mup_r.p;
+    if (half) {
+        MP_CUDA(ctx, ensure(ctx->scale, (size_t)d * sizeof(double)));
+        MP_CUDA(ctx, ensure(ctx->maxbits, (size_t)d * 2 * sizeof(unsigned long long)));
+        MP_CUDA(ctx, ensure(ctx->flat, (size_t)n * d * 3 * 2));
+        pp.scale = (double*)ctx->scale.p; pp.maxbits = (unsigned long long*)ctx->maxbits.p; pp.flat = ctx->flat.p;
+    }
+    Buf* series_bufs[2][5] = {{&ctx->st_q, &ctx->stp_q, &ctx->mu_q, &ctx->mup_q, &ctx->tw_q},
+                              {&ctx->st_r, &ctx->stp_r, &ctx->mu_r, &ctx->mup_r, &ctx->tw_r}};
+    for (int sidx = 0; sidx < (self ? 1 : 2); ++sidx) {
+        Buf** B = series_bufs[sidx];
+        MP_CUDA(ctx, ensure(*B[0], (size_t)n * d * sb));
+        if (half) MP_CUDA(ctx, ensure(*B[1], (size_t)n * d * sb));
+        MP_CUDA(ctx, ensure(*B[2], (size_t)n * d * tb));
+        MP_CUDA(ctx, ensure(*B[3], (size_t)n * Dp * tb));
+        MP_CUDA(ctx, ensure(*B[4], (size_t)L * Dp * tb));
+        pp.T = sidx == 0 ? dT : dTr;
+        pp.st = B[0]->p; pp.st_pair = B[1]->p; pp.mu = B[2]->p; pp.mup = B[3]->p; pp.tw = B[4]->p;
         MP_CUDA(ctx, mpk::launch_precompute(prec, pp, s));
     }
 
-    // keys
+    // keys (FP16 / Mixed use the FP32 key format: float bits of the half-precision sum)
     const size_t kb = (size_t)n * d * (prec == MP_FP64 ? 16 : 8);
     MP_CUDA(ctx, ensure(ctx->keys, kb));
     MP_CUDA(ctx, mpk::launch_init_keys(prec, ctx->keys.p, n * d, s));
@@ -209,6 +217,7 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
             mpk::MainParams mp{};
             mp.st_q = ctx->st_q.p;
             mp.st_r = self ? ctx->st_q.p : ctx->st_r.p;
+            if (half) mp.st_r = self ? ctx->stp_q.p : ctx->stp_r.p;   // columns: pair format
             mp.tw_q = ctx->tw_q.p;
             mp.tw_r = self ? ctx->tw_q.p : ctx->tw_r.p;
             mp.mu_q = ctx->mup_q.p;
@@ -273,7 +282,7 @@ void mp_free(mp_ctx* ctx) {
     cudaSetDevice(ctx->device);
     Buf* bufs[] = {&ctx->dT, &ctx->dTr, &ctx->st_q, &ctx->st_r, &ctx->tw_q, &ctx->tw_r, &ctx->mu_q,
                    &ctx->mu_r, &ctx->mup_q, &ctx->mup_r, &ctx->nrm, &ctx->keys, &ctx->ext, &ctx->seg, &ctx->counter, &ctx->dP,
-                   &ctx->dI, &ctx->flag};
+                   &ctx->dI, &ctx->flag, &ctx->stp_q, &ctx->stp_r, &ctx->scale, &ctx->maxbits, &ctx->flat};
     for (Buf* b : bufs) release(*b);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
     if (ctx->ev1) cudaEventDestroy(ctx->ev1);

@@ -1,0 +1,455 @@
+#pragma once
+// mp_diag16.cuh -- the fused diagonal kernel in half precision (FP16 and Mixed modes,
+// PAPER.md Fig. 1 table, Sec. III-C: "FP16 for storage and computation";
+// Mixed differs only in a FP32 precalculation, done by the precompute kernels).
+//
+// Same structure as mp_diag (mp_diag.cuh): warp tiles of consecutive diagonals, staggered
+// lane-cells, per-warp shared-memory rings staged by cp.async one batch ahead, filtered
+// min/argmin with a warp-shuffle slow path and packed-key merges.  Differences:
+//   * a lane-cell is a PAIR of adjacent diagonals (delta, delta+1) packed into __half2, so
+//     every FMA / min / max / compare of the main loop processes two cells (HFMA2, HMNMX2);
+//   * row ring entries hold duplicated half2 (x, x); column ring entries hold the pair
+//     (x_c, x_{c+1}) (precomputed in global memory), so one LDS.128 feeds both cells;
+//   * the authoritative running best per (position, rank) is an FP32 value (exact: it is a
+//     half converted to float) + index in separate arrays; the half2 thresholds in the ring
+//     are filter copies refreshed after staging and on updates.
+// Keys, finalize and the multi-GPU merge are the FP32 ones (float bits << 32 | j).
+#include <cuda_fp16.h>
+#include "mp_diag.cuh"
+
+namespace mpk {
+
+template <> struct PT<__half2> {
+    static __device__ __forceinline__ __half2 vmin(__half2 a, __half2 b) { return __hmin2(a, b); }
+    static __device__ __forceinline__ __half2 vmax(__half2 a, __half2 b) { return __hmax2(a, b); }
+};
+
+struct alignas(16) H4 { __half2 x, y, z, w; };  // (df, dg, a, threshold) for a cell pair
+
+template <int DL, int G> struct SmemH {
+    using Gm = Geo<G, 2>;
+    static constexpr int D = DL * G;
+    // rings: H4 entries + authoritative best (float value, u32 index) per (plane, slot)
+    static constexpr size_t ring_bytes =
+        (((size_t)D * (Gm::PSR + Gm::PSC) * (sizeof(H4) + 8)) + 15) & ~(size_t)15;
+    static constexpr size_t flag_bytes = ((Gm::RING_R + Gm::RING_C) * 4 + 15) & ~(size_t)15;
+    static constexpr size_t bytes_per_warp = ring_bytes + flag_bytes + (size_t)DL * 32 * sizeof(__half2);
+    static constexpr int WPB = bytes_per_warp * 4 <= 112 * 1024 ? 4 : bytes_per_warp * 2 <= 112 * 1024 ? 2 : 1;
+};
+
+template <int DL, int G, bool SELF, bool MIXED>
+__global__ void __launch_bounds__(128)
+mp_diag_h(const MainParams p) {
+    using Gm = Geo<G, 2>;
+    using SM = SmemH<DL, G>;
+    using TS = typename std::conditional<MIXED, float, __half>::type;  // seed operand type
+    constexpr int CA = Gm::CA, RA = Gm::RA, CW = Gm::CW, D = DL * G;
+    constexpr int PSR = Gm::PSR, PSC = Gm::PSC, SB = Gm::SB;
+
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    unsigned char* wbase = smem_raw + (size_t)warp * SM::bytes_per_warp;
+    H4* rowv = reinterpret_cast<H4*>(wbase);
+    H4* colv = rowv + (size_t)D * PSR;
+    float* rowb = reinterpret_cast<float*>(colv + (size_t)D * PSC);
+    float* colb = rowb + (size_t)D * PSR;
+    unsigned* rowi = reinterpret_cast<unsigned*>(colb + (size_t)D * PSC);
+    unsigned* coli = rowi + (size_t)D * PSR;
+    unsigned* rowdirty = reinterpret_cast<unsigned*>(wbase + SM::ring_bytes);
+    unsigned* coldirty = rowdirty + Gm::RING_R;
+    __half2* ssc = reinterpret_cast<__half2*>(wbase + SM::ring_bytes + SM::flag_bytes);
+
+    const H4* __restrict__ st_q = reinterpret_cast<const H4*>(p.st_q);   // row format (x, x)
+    const H4* __restrict__ st_r = reinterpret_cast<const H4*>(p.st_r);   // pair format (x_c, x_c+1)
+    const TS* __restrict__ tw_q = reinterpret_cast<const TS*>(p.tw_q);
+    const TS* __restrict__ tw_r = reinterpret_cast<const TS*>(p.tw_r);
+    const TS* __restrict__ mu_q = reinterpret_cast<const TS*>(p.mu_q);
+    const TS* __restrict__ mu_r = reinterpret_cast<const TS*>(p.mu_r);
+    unsigned long long* keys = reinterpret_cast<unsigned long long*>(p.keys);
+
+    const long long n = p.n;
+    const int d = p.d, m = p.m, H = p.H;
+    const int n32 = (int)n;
+    const __half2 two_m = __float2half2_rn((float)(2 * m));
+    const float FINF = __int_as_float(0x7f800000);
+    const __half HINF = __ushort_as_half(0x7c00), HNINF = __ushort_as_half(0xfc00);
+
+    const int lc = lane >> Gm::LOG_G, g = lane & (G - 1);
+    const int a = lc >> Gm::LOG_CA, c = lc & (CA - 1);
+    unsigned gmask_row = 0, gmask_col = 0;
+#pragma unroll
+    for (int cc = 0; cc < CA; ++cc) gmask_row |= 1u << (((a * CA + cc) << Gm::LOG_G) + g);
+#pragma unroll
+    for (int aa = 0; aa < RA; ++aa) gmask_col |= 1u << (((aa * CA + c) << Gm::LOG_G) + g);
+
+    // ---- staging: stats by cp.async (12 B of the 16 B entry), authoritative best from the
+    // merge key (value half -> float, index half -> u32); the half2 filter copies of the
+    // thresholds are written by fixup() once the copies have landed.
+    auto stage = [&](bool is_row, int base, int p_lo, int p_hi) {
+        const int cnt = p_hi - p_lo;
+        if (cnt <= 0) return;
+        H4* buf = is_row ? rowv : colv;
+        float* bb = is_row ? rowb : colb;
+        unsigned* ib = is_row ? rowi : coli;
+        unsigned* dflag = is_row ? rowdirty : coldirty;
+        const int ps = is_row ? PSR : PSC;
+        const H4* __restrict__ st = is_row ? st_q : st_r;
+        const bool want_thr = is_row || SELF;
+        for (int e = lane; e < cnt * D; e += 32) {
+            const int pi = e / D, pl = e - pi * D;
+            const int pos = base + p_lo + pi;
+            if (pos < 0 || pos >= n32) continue;
+            const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
+            if (pl == 0) dflag[sl] = 0;
+            H4* dst = &buf[pl * ps + sl];
+            if (pl < d) {
+                const H4* src = st + (size_t)pos * d + pl;
+                cp_async8(dst, src);
+                cp_async4(&dst->z, &src->z);
+            } else {  // padded dimension: a = +inf with QT = -1 gives D = +inf
+                dst->x = __half2half2(__float2half(0.f));
+                dst->y = dst->x;
+                dst->z = __half2half2(HINF);
+            }
+            const int rk = rank_of_plane<DL, G>(pl);
+            if (rk < d && want_thr) {
+                const unsigned long long* kp = keys + (size_t)pos * d + rk;
+                cp_async4(&bb[pl * ps + sl], reinterpret_cast<const char*>(kp) + 4);
+                cp_async4(&ib[pl * ps + sl], kp);
+            } else {
+                bb[pl * ps + sl] = -FINF;
+                ib[pl * ps + sl] = 0x7fffffffu;
+            }
+        }
+    };
+    // thresholds (half) from the landed authoritative bests: row (t, t); column c -> low half
+    // of slot c and high half of slot c-1 (the pair (c-1, c))
+    auto fixup = [&](bool is_row, int base, int p_lo, int p_hi) {
+        const int cnt = p_hi - p_lo;
+        if (cnt <= 0) return;
+        H4* buf = is_row ? rowv : colv;
+        const float* bb = is_row ? rowb : colb;
+        const int ps = is_row ? PSR : PSC;
+        for (int e = lane; e < cnt * D; e += 32) {
+            const int pi = e / D, pl = e - pi * D;
+            const int pos = base + p_lo + pi;
+            if (pos < 0 || pos >= n32) continue;
+            if (is_row) {
+                const int sl = Gm::srow(pos);
+                buf[pl * ps + sl].w = __half2half2(__float2half_rn(bb[pl * ps + sl]));
+            } else {
+                const int sl = Gm::scol(pos);
+                const __half h = __float2half_rn(bb[pl * ps + sl]);
+                reinterpret_cast<__half*>(&buf[pl * ps + sl].w)[0] = h;
+                reinterpret_cast<__half*>(&buf[pl * ps + Gm::scol(pos - 1)].w)[1] = h;
+            }
+        }
+    };
+    auto evict = [&](bool is_row, int base, int p_lo, int p_hi) {
+        if (!is_row && !SELF) return;
+        const int cnt = p_hi - p_lo;
+        if (cnt <= 0) return;
+        const float* bb = is_row ? rowb : colb;
+        const unsigned* ib = is_row ? rowi : coli;
+        const unsigned* dflag = is_row ? rowdirty : coldirty;
+        const int ps = is_row ? PSR : PSC;
+        bool any = false;
+        for (int pi = lane; pi < cnt; pi += 32) {
+            const int pos = base + p_lo + pi;
+            if (pos >= 0 && pos < n32) any |= dflag[is_row ? Gm::srow(pos) : Gm::scol(pos)] != 0;
+        }
+        if (!__any_sync(FULL, any)) return;
+        for (int e = lane; e < cnt * D; e += 32) {
+            const int pi = e / D, pl = e - pi * D;
+            const int pos = base + p_lo + pi;
+            if (pos < 0 || pos >= n32) continue;
+            const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
+            if (dflag[sl] == 0) continue;
+            const int rk = rank_of_plane<DL, G>(pl);
+            if (rk >= d) continue;
+            const unsigned ix = ib[pl * ps + sl];
+            if (ix & DIRTY) KeyOps<float>::merge(keys + (size_t)pos * d + rk, bb[pl * ps + sl], ix & ~DIRTY);
+        }
+    };
+
+    for (;;) {
+        long long t = 0;
+        if (lane == 0) t = (long long)atomicAdd(p.counter, 1ull);
+        t = __shfl_sync(FULL, t, 0);
+        if (t >= p.t_count) break;
+        t += p.t_begin;
+        long long lo_b = 0, hi_b = p.nb;
+        while (hi_b - lo_b > 1) {
+            const long long mid = (lo_b + hi_b) >> 1;
+            if (__ldg(&p.seg_prefix[mid]) <= t) lo_b = mid; else hi_b = mid;
+        }
+        const long long b = lo_b;
+        const long long delta0 = p.delta_lo + b * Gm::NC;
+        const long long delta1 = min(delta0 + Gm::NC - 1, p.delta_hi);
+        const long long rlo = max(0ll, -delta1), rhi = min(n, n - max(delta0, 0ll));
+        const long long q = rlo / H + (t - __ldg(&p.seg_prefix[b]));
+        const long long r0 = max(q * H, rlo), r1 = min((q + 1) * H, rhi);
+
+        long long delta[2], lo[2], hi[2];
+        int dlt[2], lo32[2], hi32[2];
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+            delta[u] = delta0 + (long long)a * CW + c * 2 + u;
+            lo[u] = max(r0, max(0ll, -delta[u]));
+            hi[u] = min(r1, n - max(delta[u], 0ll));
+            if (delta[u] > p.delta_hi) hi[u] = lo[u];
+            dlt[u] = (int)delta[u]; lo32[u] = (int)lo[u]; hi32[u] = (int)hi[u];
+        }
+
+        // seeds at each cell's first row: Mixed -> FP32 operands and compensated FP32
+        // accumulation rounded to half (FP32 precalc); FP16 -> half arithmetic throughout
+        // seeds at the pair's first row (both cells start at row r0 except at diagonal starts):
+        // Mixed -> FP32 operands and FP32 accumulation rounded to half (the FP32 precalc);
+        // FP16 -> half arithmetic.  The row window is shared by the pair and the second cell's
+        // column window is the first one shifted by one position.
+        __half2 QT[DL];
+        {
+            using TA = typename std::conditional<MIXED, float, __half>::type;
+            const bool ok0 = lo[0] < hi[0], ok1 = lo[1] < hi[1];
+            const bool same = ok0 && ok1 && lo[0] == lo[1];
+            TA acc0[DL], acc1[DL];
+#pragma unroll
+            for (int kk = 0; kk < DL; ++kk) { acc0[kk] = (TA)0.f; acc1[kk] = (TA)0.f; }
+#pragma unroll 1
+            for (int u = 0; u < (same ? 1 : 2); ++u) {
+                const bool ok = u == 0 ? ok0 : ok1;
+                if (!ok) continue;
+                const long long i0 = lo[u], j0 = lo[u] + delta[u];
+                TA mq[DL], mr0[DL], mr1[DL];
+#pragma unroll
+                for (int kk = 0; kk < DL; ++kk) {
+                    mq[kk] = mu_q[i0 * D + kk * G + g];
+                    mr0[kk] = mu_r[j0 * D + kk * G + g];
+                    mr1[kk] = same ? mu_r[(j0 + 1) * D + kk * G + g] : mr0[kk];
+                }
+                TA xr_prev[DL];
+#pragma unroll
+                for (int kk = 0; kk < DL; ++kk) xr_prev[kk] = tw_r[j0 * D + kk * G + g];
+#pragma unroll 2
+                for (int tt = 0; tt < m; ++tt) {
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) {
+                        const TA xq = tw_q[(i0 + tt) * D + kk * G + g];
+                        const TA xr = xr_prev[kk];
+                        if (same) {
+                            const TA xn = tw_r[(j0 + tt + 1) * D + kk * G + g];
+                            acc0[kk] = acc0[kk] + (xq - mq[kk]) * (xr - mr0[kk]);
+                            acc1[kk] = acc1[kk] + (xq - mq[kk]) * (xn - mr1[kk]);
+                            xr_prev[kk] = xn;
+                        } else {
+                            TA& acc = u == 0 ? acc0[kk] : acc1[kk];
+                            acc = acc + (xq - mq[kk]) * (xr - mr0[kk]);
+                            xr_prev[kk] = tw_r[(j0 + tt + 1) * D + kk * G + g];
+                        }
+                    }
+                }
+            }
+#pragma unroll
+            for (int kk = 0; kk < DL; ++kk) {
+                const bool pad = (kk * G + g) >= d;
+                const float v0 = pad ? -1.f : (float)acc0[kk], v1 = pad ? -1.f : (float)acc1[kk];
+                QT[kk] = __floats2half2_rn(v0, v1);
+            }
+        }
+
+        const int nrows = (int)(r1 - r0);
+        const int s_end = nrows + CW * (RA - 1);
+        const int R0 = (int)r0, C0 = (int)(r0 + delta0);
+        int row_in = min(SB, nrows), col_in = min(SB, s_end) + CW;  // pairs need column c+1's slot too
+        int row_out = 0, col_out = 0;
+        int fx_r0 = 0, fx_r1 = row_in, fx_c0 = 0, fx_c1 = col_in;
+        stage(true, R0, 0, row_in);
+        stage(false, C0, 0, col_in);
+        cp_async_commit();
+        cp_async_wait_all();
+        __syncwarp();
+        fixup(true, R0, fx_r0, fx_r1);
+        fixup(false, C0, fx_c0, fx_c1);
+        fx_r0 = fx_r1; fx_c0 = fx_c1;
+        __syncwarp();
+
+        auto step = [&](int s) {
+            const int row = R0 + s - CW * a;
+            const int sr = Gm::srow(row);
+            const int col0 = row + dlt[0];
+            const int scn = Gm::scol(col0);
+            bool active[2], upd[2];
+#pragma unroll
+            for (int u = 0; u < 2; ++u) {
+                active[u] = row >= lo32[u] && row < hi32[u];
+                upd[u] = row > lo32[u] && row < hi32[u];
+            }
+            __half2 S[DL], tr[DL], tc[DL];
+            if (upd[0] == upd[1]) {
+#pragma unroll
+                for (int kk = 0; kk < DL; ++kk) {
+                    const int pl = kk * G + g;
+                    const H4 R = rowv[pl * PSR + sr];
+                    const H4 C = colv[pl * PSC + scn];
+                    if (upd[0]) QT[kk] = __hfma2(R.x, C.y, __hfma2(C.x, R.y, QT[kk]));   // Eq. (1)
+                    S[kk] = h2sqrt(__habs2(__hfma2(__hneg2(QT[kk]), __hmul2(R.z, C.z), two_m)));
+                    tr[kk] = R.w;
+                    tc[kk] = C.w;
+                }
+            } else {  // the two cells of the pair are at different phases (tile / diagonal start)
+                const __half2 msk = __halves2half2(__float2half(upd[0] ? 1.f : 0.f), __float2half(upd[1] ? 1.f : 0.f));
+#pragma unroll
+                for (int kk = 0; kk < DL; ++kk) {
+                    const int pl = kk * G + g;
+                    const H4 R = rowv[pl * PSR + sr];
+                    const H4 C = colv[pl * PSC + scn];
+                    QT[kk] = __hfma2(msk, __hfma2(R.x, C.y, __hmul2(C.x, R.y)), QT[kk]);
+                    S[kk] = h2sqrt(__habs2(__hfma2(__hneg2(QT[kk]), __hmul2(R.z, C.z), two_m)));
+                    tr[kk] = R.w;
+                    tc[kk] = C.w;
+                }
+            }
+            sort_net<__half2, DL>(S);                                              // Eq. (2)
+            if (G > 1) lane_merge<__half2, DL, G>(S, g);
+#pragma unroll
+            for (int kk = 1; kk < DL; ++kk) S[kk] = __hadd2(S[kk], S[kk - 1]);     // Eq. (2)
+            if (G > 1) {
+                __half2 tot = S[DL - 1];
+#pragma unroll
+                for (int dd = 1; dd < G; dd <<= 1) {
+                    const __half2 y = __shfl_up_sync(FULL, tot, dd, G);
+                    if (g >= dd) tot = __hadd2(tot, y);
+                }
+                __half2 excl = __shfl_up_sync(FULL, tot, 1, G);
+                if (g == 0) excl = __float2half2_rn(0.f);
+#pragma unroll
+                for (int kk = 0; kk < DL; ++kk) S[kk] = __hadd2(S[kk], excl);
+            }
+            unsigned hm[4] = {0u, 0u, 0u, 0u};
+#pragma unroll
+            for (int kk = 0; kk < DL; ++kk) {
+                hm[kk & 3] |= __hle2_mask(S[kk], tr[kk]);
+                if (SELF) hm[kk & 3] |= __hle2_mask(S[kk], tc[kk]);
+            }
+            const unsigned hmask = (hm[0] | hm[1]) | (hm[2] | hm[3]);
+            const bool hit = ((hmask & 0xffffu) && active[0]) || ((hmask >> 16) && active[1]);
+            if (__any_sync(FULL, hit)) {
+#pragma unroll
+                for (int kk = 0; kk < DL; ++kk) {
+                    __half2 v = S[kk];
+                    if (!active[0]) v = __halves2half2(HINF, __high2half(v));
+                    if (!active[1]) v = __halves2half2(__low2half(v), HINF);
+                    ssc[kk * 32 + lane] = v;
+                }
+                __syncwarp();
+#pragma unroll 1
+                for (int kk = 0; kk < DL; ++kk) {
+                    const int pl = kk * G + g;
+                    const __half2 vh = ssc[kk * 32 + lane];
+                    const float v[2] = {__low2float(vh), __high2float(vh)};
+                    float vr = fminf(v[0], v[1]);
+#pragma unroll
+                    for (int bit = 0; bit < Gm::LOG_CA; ++bit)
+                        vr = fminf(vr, __shfl_xor_sync(FULL, vr, 1 << (bit + Gm::LOG_G)));
+                    const bool mine = v[0] == vr || v[1] == vr;
+                    const unsigned eqr = __ballot_sync(FULL, mine) & gmask_row;
+                    if (vr < FINF && lane == __ffs(eqr) - 1) {
+                        const int j = (v[0] == vr) ? col0 : col0 + 1;          // lowest column first
+                        const int ix = pl * PSR + sr;
+                        const float cur = rowb[ix];
+                        const unsigned ci = rowi[ix] & ~DIRTY;
+                        if (vr < cur || (vr == cur && (unsigned)j < ci)) {
+                            rowb[ix] = vr;
+                            rowi[ix] = (unsigned)j | DIRTY;
+                            rowv[ix].w = __float2half2_rn(vr);
+                            rowdirty[sr] = 1;
+                        }
+                    }
+                    if (SELF) {
+#pragma unroll
+                        for (int u = 0; u < 2; ++u) {
+                            float vc = v[u];
+#pragma unroll
+                            for (int bit = 0; bit < 5 - Gm::LOG_G - Gm::LOG_CA; ++bit)
+                                vc = fminf(vc, __shfl_xor_sync(FULL, vc, 1 << (bit + Gm::LOG_G + Gm::LOG_CA)));
+                            const unsigned eqc = __ballot_sync(FULL, v[u] == vc) & gmask_col;
+                            if (vc < FINF && eqc != 0 && lane == 31 - __clz(eqc)) {
+                                const int colu = col0 + u;
+                                const int scu = Gm::scol(colu);
+                                const int ix = pl * PSC + scu;
+                                const float cur = colb[ix];
+                                const unsigned ci = coli[ix] & ~DIRTY;
+                                if (vc < cur || (vc == cur && (unsigned)row < ci)) {
+                                    colb[ix] = vc;
+                                    coli[ix] = (unsigned)row | DIRTY;
+                                    const __half h = __float2half_rn(vc);
+                                    reinterpret_cast<__half*>(&colv[ix].w)[0] = h;
+                                    reinterpret_cast<__half*>(&colv[pl * PSC + Gm::scol(colu - 1)].w)[1] = h;
+                                    coldirty[scu] = 1;
+                                }
+                            }
+                        }
+                    }
+                }
+                __syncwarp();
+            }
+        };
+
+        for (int s0 = 0; s0 < s_end; s0 += SB) {
+            const int rx = min(max(s0 - CW * (RA - 1), 0), nrows);
+            evict(true, R0, row_out, rx);
+            row_out = rx;
+            evict(false, C0, col_out, s0);
+            col_out = s0;
+            const int nxt = min(s0 + 2 * SB, s_end);
+            const int r_need = min(nxt, nrows), c_need = nxt + CW;
+            stage(true, R0, row_in, r_need);
+            stage(false, C0, col_in, c_need);
+            fx_r1 = max(row_in, r_need);
+            fx_c1 = max(col_in, c_need);
+            row_in = fx_r1;
+            col_in = fx_c1;
+            cp_async_commit();
+            const int s1 = min(s0 + SB, s_end);
+#pragma unroll 1
+            for (int ss = s0; ss < s1; ++ss) step(ss);
+            cp_async_wait_all();
+            __syncwarp();
+            fixup(true, R0, fx_r0, fx_r1);
+            fixup(false, C0, fx_c0, fx_c1);
+            fx_r0 = fx_r1;
+            fx_c0 = fx_c1;
+            __syncwarp();
+        }
+        evict(true, R0, row_out, nrows);
+        evict(false, C0, col_out, col_in);
+        __syncwarp();
+    }
+}
+
+template <int DL, int G, bool SELF, bool MIXED> struct InstH {
+    static size_t smem() { return SmemH<DL, G>::bytes_per_warp * SmemH<DL, G>::WPB; }
+    static int warps_per_block() { return SmemH<DL, G>::WPB; }
+    static cudaError_t launch(const MainParams& p, int grid, cudaStream_t s);
+    static int blocks_per_sm();
+};
+
+#ifdef MP_DIAG_IMPL
+template <int DL, int G, bool SELF, bool MIXED>
+cudaError_t InstH<DL, G, SELF, MIXED>::launch(const MainParams& p, int grid, cudaStream_t s) {
+    const size_t sm = smem();
+    cudaError_t e = cudaFuncSetAttribute(mp_diag_h<DL, G, SELF, MIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e != cudaSuccess) return e;
+    mp_diag_h<DL, G, SELF, MIXED><<<grid, SmemH<DL, G>::WPB * 32, sm, s>>>(p);
+    return cudaGetLastError();
+}
+template <int DL, int G, bool SELF, bool MIXED> int InstH<DL, G, SELF, MIXED>::blocks_per_sm() {
+    const size_t sm = smem();
+    cudaFuncSetAttribute(mp_diag_h<DL, G, SELF, MIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    int nb = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mp_diag_h<DL, G, SELF, MIXED>, SmemH<DL, G>::WPB * 32, sm);
+    return nb;
+}
+#endif
+
+}  // namespace mpk

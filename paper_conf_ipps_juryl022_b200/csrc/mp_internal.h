@@ -35,6 +35,11 @@ struct PreParams {
     double* nrm64;
     long long n;
     int d, m;
+    // FP16 / Mixed only
+    void* st_pair;      // out stats in pair format [pos][dim] (x_pos, x_pos+1) half2 x 4
+    double* scale;      // scratch [d]: exact power-of-two per-dimension scale (reading G16)
+    unsigned long long* maxbits;  // scratch [2 d]: max window norm, max |x| (double bits)
+    void* flat;         // scratch [3][pos][dim] half: df, dg, a
 };
 
 // Precision codes match mp_precision.

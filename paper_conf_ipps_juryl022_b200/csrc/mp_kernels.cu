@@ -1,7 +1,7 @@
 // mp_kernels.cu -- precompute, key and finalize kernels + dispatch of the fused kernel.
 // The fused diagonal kernel itself lives in mp_diag.cuh (instantiated in inst_*.cu so
 // the heavy template variants compile in parallel).
-#include "mp_diag.cuh"
+#include "mp_diag16.cuh"
 
 namespace mpk {
 
@@ -85,6 +85,148 @@ __global__ void pre_pm(const PreParams p) {
     if (t < n) mup[gid] = dim < d ? reinterpret_cast<const T*>(p.mu)[(long long)dim * n + t] : (T)0;
 }
 
+// ------------------------------------------------------------------ precompute, FP16 / Mixed
+// Reading G16: an exact power-of-two scale s_k per dimension keeps the half-precision
+// window energies (QT, norm^2) <= 2^14 (and, for FP16, the window sums <= 2^14); z-normalised
+// distances are invariant under it (pinned in tests/test_oracle.py).
+__global__ void pre_scale_max(const PreParams p) {
+    const long long n = p.n, L = p.n + p.m - 1;
+    const int d = p.d, m = p.m;
+    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (gid >= n * d) return;
+    const int dim = (int)(gid / n);
+    const long long pos = gid % n;
+    const double* x = p.T + (long long)dim * L + pos;
+    double s = 0, amax = 0;
+    for (int t = 0; t < m; ++t) { s += x[t]; amax = fmax(amax, fabs(x[t])); }
+    const double mu = s / m;
+    double q = 0;
+    for (int t = 0; t < m; ++t) q = fma(x[t] - mu, x[t] - mu, q);
+    atomicMax(&p.maxbits[dim], (unsigned long long)__double_as_longlong(sqrt(q)));
+    atomicMax(&p.maxbits[d + dim], (unsigned long long)__double_as_longlong(amax));
+}
+__global__ void pre_scale_pick(const PreParams p, int pure16) {
+    const int dim = blockIdx.x * blockDim.x + threadIdx.x;
+    if (dim >= p.d) return;
+    const double nmax = __longlong_as_double((long long)p.maxbits[dim]);
+    const double amax = __longlong_as_double((long long)p.maxbits[p.d + dim]);
+    int e = 0;
+    if (nmax > 0) e = (int)floor(log2(128.0 / nmax));
+    if (pure16 && amax > 0) e = min(e, (int)floor(log2(16384.0 / ((double)p.m * amax))));
+    e = max(-60, min(60, e));
+    p.scale[dim] = ldexp(1.0, e);
+}
+template <class T>  // T = float (Mixed: FP32 precalc) or __half (FP16: half precalc)
+__global__ void pre_stats_h(const PreParams p) {
+    const long long n = p.n, L = p.n + p.m - 1;
+    const int d = p.d, m = p.m;
+    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (gid >= n * d) return;
+    const int dim = (int)(gid / n);
+    const long long pos = gid % n;
+    const double sc = p.scale[dim];
+    const double* x = p.T + (long long)dim * L + pos;
+    T mu, nr;
+    if constexpr (sizeof(T) == 4) {  // compensated, as in FP32 mode
+        float s = 0, c = 0;
+        for (int t = 0; t < m; ++t) { const float y = (float)(sc * x[t]) - c; const float tt = s + y; c = (tt - s) - y; s = tt; }
+        mu = s / (float)m;
+        float q = 0;
+        c = 0;
+        for (int t = 0; t < m; ++t) {
+            const float cx = (float)(sc * x[t]) - mu;
+            const float y = cx * cx - c; const float tt = q + y; c = (tt - q) - y; q = tt;
+        }
+        nr = sqrtf(q);
+    } else {  // FP16 mode: plain half arithmetic (the paper's uncompensated FP16 precalc)
+        __half s = __float2half(0.f);
+        for (int t = 0; t < m; ++t) s = __hadd(s, __double2half(sc * x[t]));
+        mu = __hdiv(s, __int2half_rn(m));
+        __half q = __float2half(0.f);
+        for (int t = 0; t < m; ++t) {
+            const __half cx = __hsub(__double2half(sc * x[t]), mu);
+            q = __hfma(cx, cx, q);
+        }
+        nr = hsqrt(q);
+    }
+    reinterpret_cast<T*>(p.mu)[(long long)dim * n + pos] = mu;
+    reinterpret_cast<T*>(p.nrm32)[(long long)dim * n + pos] = nr;   // typed scratch
+}
+template <class T>
+__global__ void pre_diff_h(const PreParams p) {
+    const long long n = p.n, L = p.n + p.m - 1;
+    const int d = p.d, m = p.m;
+    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (gid >= n * d) return;
+    const long long pos = gid / d;
+    const int dim = (int)(gid % d);
+    const double sc = p.scale[dim];
+    const double* x = p.T + (long long)dim * L;
+    const T* mu = reinterpret_cast<const T*>(p.mu) + (long long)dim * n;
+    const T nr = reinterpret_cast<const T*>(p.nrm32)[(long long)dim * n + pos];
+    __half* flat = reinterpret_cast<__half*>(p.flat);
+    float df = 0, dg = 0, av;
+    if constexpr (sizeof(T) == 4) {
+        if (pos > 0) {
+            const float xl = (float)(sc * x[pos + m - 1]), xf = (float)(sc * x[pos - 1]);
+            df = (xl - xf) / 2.f;
+            dg = (xl - mu[pos]) + (xf - mu[pos - 1]);
+        }
+        av = nr > 0.f ? sqrtf((float)(2 * m)) / nr : 0.f;
+    } else {
+        if (pos > 0) {
+            const __half xl = __double2half(sc * x[pos + m - 1]), xf = __double2half(sc * x[pos - 1]);
+            df = __half2float(__hdiv(__hsub(xl, xf), __float2half(2.f)));
+            dg = __half2float(__hadd(__hsub(xl, mu[pos]), __hsub(xf, mu[pos - 1])));
+        }
+        av = __half2float(nr) > 0.f ? __half2float(__hdiv(hsqrt(__int2half_rn(2 * m)), nr)) : 0.f;
+    }
+    av = fminf(av, 65504.f);  // finite half (near-flat windows)
+    const long long o = pos * d + dim;
+    flat[o] = __float2half_rn(df);
+    flat[n * d + o] = __float2half_rn(dg);
+    flat[2 * n * d + o] = __float2half_rn(av);
+}
+// row format (x, x) and pair format (x_pos, x_pos+1) H4 entries for the half2 kernel
+__global__ void pre_fmt_h(const PreParams p) {
+    const long long n = p.n;
+    const int d = p.d;
+    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (gid >= n * d) return;
+    const long long pos = gid / d;
+    const __half* f = reinterpret_cast<const __half*>(p.flat);
+    const long long nd = n * d;
+    const __half z = __float2half(0.f);
+    H4 r, q;
+    r.x = __half2half2(f[gid]); r.y = __half2half2(f[nd + gid]); r.z = __half2half2(f[2 * nd + gid]);
+    r.w = __half2half2(z);
+    const bool nx = pos + 1 < n;
+    q.x = __halves2half2(f[gid], nx ? f[gid + d] : z);
+    q.y = __halves2half2(f[nd + gid], nx ? f[nd + gid + d] : z);
+    q.z = __halves2half2(f[2 * nd + gid], nx ? f[2 * nd + gid + d] : z);
+    q.w = __half2half2(z);
+    reinterpret_cast<H4*>(p.st)[gid] = r;
+    reinterpret_cast<H4*>(p.st_pair)[gid] = q;
+}
+template <class T>
+__global__ void pre_pm_h(const PreParams p) {
+    const long long n = p.n, L = p.n + p.m - 1;
+    const int d = p.d, Dp = p.Dp;
+    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (gid >= L * Dp) return;
+    const long long t = gid / Dp;
+    const int dim = (int)(gid % Dp);
+    T* tw = reinterpret_cast<T*>(p.tw);
+    T* mup = reinterpret_cast<T*>(p.mup);
+    if (dim < d) {
+        const double v = p.scale[dim] * p.T[(long long)dim * L + t];
+        if constexpr (sizeof(T) == 4) tw[gid] = (float)v; else tw[gid] = __double2half(v);
+    } else {
+        tw[gid] = (T)0.f;
+    }
+    if (t < n) mup[gid] = dim < d ? reinterpret_cast<const T*>(p.mu)[(long long)dim * n + t] : (T)0.f;
+}
+
 // ------------------------------------------------------------------ keys
 __global__ void init_keys32(unsigned long long* k, long long count) {
     const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
@@ -150,7 +292,12 @@ Variant pick_variant(int prec, int d) {
     int dp = 1;
     while (dp < d) dp <<= 1;
     Variant v;
-    if (prec == P64) {
+    if (prec == P16 || prec == PMIX) {  // half2: a lane-cell is a pair of diagonals
+        if (dp <= 8) { v.DL = dp; v.G = 1; }
+        else if (dp <= 256) { v.DL = 8; v.G = dp / 8; }
+        else { v.DL = dp / 32; v.G = 32; }
+        v.W = 2;
+    } else if (prec == P64) {
         if (dp <= 16) { v.DL = dp; v.G = 1; v.W = dp <= 8 ? 2 : 1; }
         else { v.DL = 16; v.G = dp / 16; v.W = 1; }
     } else {
@@ -184,8 +331,25 @@ static long long dispatch_t(int op, int DL, int G, int W, const MainParams* p, i
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
 }
 
+template <bool SELF, bool MIXED>
+static long long dispatch_h(int op, int DL, int G, const MainParams* p, int grid, cudaStream_t s) {
+#define MP_HCASE(dl, g)                                                                    \
+    if (DL == dl && G == g) {                                                              \
+        if (op == 0) return (long long)InstH<dl, g, SELF, MIXED>::smem();                  \
+        if (op == 1) return (long long)InstH<dl, g, SELF, MIXED>::launch(*p, grid, s);     \
+        if (op == 3) return InstH<dl, g, SELF, MIXED>::warps_per_block();                  \
+        return InstH<dl, g, SELF, MIXED>::blocks_per_sm();                                 \
+    }
+    MP_HCASE(1, 1) MP_HCASE(2, 1) MP_HCASE(4, 1) MP_HCASE(8, 1)
+    MP_HCASE(8, 2) MP_HCASE(8, 4) MP_HCASE(8, 8) MP_HCASE(8, 16) MP_HCASE(8, 32) MP_HCASE(16, 32) MP_HCASE(32, 32)
+#undef MP_HCASE
+    return op == 1 ? (long long)cudaErrorInvalidValue : 0;
+}
+
 static long long dispatch(int op, int prec, bool self, int d, const MainParams* p, int grid, cudaStream_t s) {
     const Variant v = pick_variant(prec, d);
+    if (prec == P16) return self ? dispatch_h<true, false>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, false>(op, v.DL, v.G, p, grid, s);
+    if (prec == PMIX) return self ? dispatch_h<true, true>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, true>(op, v.DL, v.G, p, grid, s);
     if (prec == P64) return self ? dispatch_t<double, true>(op, v.DL, v.G, v.W, p, grid, s) : dispatch_t<double, false>(op, v.DL, v.G, v.W, p, grid, s);
     if (prec == P32) return self ? dispatch_t<float, true>(op, v.DL, v.G, v.W, p, grid, s) : dispatch_t<float, false>(op, v.DL, v.G, v.W, p, grid, s);
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
@@ -210,7 +374,20 @@ cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s) {
         pre_diff<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
         pre_pm<float><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
     } else {
-        return cudaErrorInvalidValue;
+        const bool mixed = prec == PMIX;
+        cudaMemsetAsync(p.maxbits, 0, 2 * p.d * sizeof(unsigned long long), s);
+        pre_scale_max<<<grid1d(cnt, 256), 256, 0, s>>>(p);
+        pre_scale_pick<<<grid1d(p.d, 128), 128, 0, s>>>(p, mixed ? 0 : 1);
+        if (mixed) {
+            pre_stats_h<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+            pre_diff_h<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+            pre_pm_h<float><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
+        } else {
+            pre_stats_h<__half><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+            pre_diff_h<__half><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+            pre_pm_h<__half><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
+        }
+        pre_fmt_h<<<grid1d(cnt, 256), 256, 0, s>>>(p);
     }
     return cudaGetLastError();
 }

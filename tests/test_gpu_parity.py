@@ -185,3 +185,66 @@ def test_invalid_arguments(ctx):
         ctx.compute(T, 1, "fp32")
     with pytest.raises(mstamp.MPError):
         ctx.compute(np.zeros((2000, 10)), 4, "fp32")
+
+
+# ---------------------------------------------------------------- FP16 / Mixed (parity unpinned)
+def _half_stats(P_or, I_or, P, I, m):
+    fin = np.isfinite(P_or)
+    rel = np.abs(P - P_or)[fin] / np.maximum(P_or[fin], 0.05 * math.sqrt(2 * m))
+    return dict(median_rel=float(np.median(rel)), p99_rel=float(np.quantile(rel, 0.99)),
+                max_rel=float(rel.max()), recall=float((I == I_or)[fin].mean()))
+
+
+@pytest.mark.parametrize("prec", ["fp16", "mixed"])
+def test_half_modes_c1(ctx, oracle_mod, c1_oracle, prec):
+    """FP16 / Mixed: no tolerance gate (parity unpinned); the
+    error vs FP64 is measured and must stay within the stated bound; the planted motif must
+    be recovered (the paper's R_embedded, L911-915) and the distance bound must hold."""
+    cfg, P, I, P2 = c1_oracle
+    m = cfg["m"]
+    Pg, Ig = ctx.compute(cfg["T"], m, prec, cfg["exclusion"])
+    st = _half_stats(P, I, Pg, Ig, m)
+    print(prec, st)
+    # stated bounds (DESIGN.md): Mixed median 2 %, p99 20 %; FP16 (half-precision precalc of an
+    # offset random walk, the paper's least accurate mode) median 20 %, p99 100 %
+    med, p99 = (0.02, 0.2) if prec == "mixed" else (0.2, 1.0)
+    assert st["median_rel"] < med and st["p99_rel"] < p99
+    assert np.all(Pg >= 0) and np.all(Pg <= 2 * math.sqrt(m) * 1.01)
+    a, b = datagen.motif_positions(cfg["n"], m)
+    for k in range(max(1, cfg["d"] // 2)):
+        assert Ig[k, a] == b and Ig[k, b] == a
+
+
+@pytest.mark.parametrize("prec", ["fp16", "mixed"])
+@pytest.mark.parametrize("shape", [(3, 700, 32, 8, 51), (16, 900, 64, 16, 52), (40, 300, 16, 4, 53)])
+def test_half_modes_shapes(ctx, oracle_mod, prec, shape):
+    d, n, m, e, seed = shape
+    T = datagen.bounded_patterns(d, n, m, seed)
+    P, I, P2 = oracle_mod.mstamp(T, m, e)
+    Pg, Ig = ctx.compute(T, m, prec, e)
+    st = _half_stats(P, I, Pg, Ig, m)
+    print(prec, shape, st)
+    assert st["median_rel"] < (0.05 if prec == "mixed" else 0.2)
+    assert np.all(np.isfinite(Pg))
+
+
+@pytest.mark.parametrize("prec", ["fp16", "mixed"])
+def test_half_modes_ab_and_bands(ctx, prec):
+    """AB-join runs; band partials merge bit-identically to the single band (FP32 key format)."""
+    from paper_conf_ipps_juryl022_b200 import mstamp
+    d, n, m = 4, 1500, 32
+    Tq, Tr = datagen.random_walk_ab(d, n, m, 54)
+    Pg, Ig = ctx.compute(Tq, m, prec, Tr=Tr)
+    assert np.all(np.isfinite(Pg)) and np.all((Ig >= 0) & (Ig < n))
+    T = torch.from_numpy(datagen.random_walk(d, n, m, 55)).cuda()
+    kw = mstamp.key_words(d, n, prec)
+    full = torch.empty(kw, dtype=torch.int64, device="cuda")
+    ctx.partial_device(T, m, full, 0, 1, prec, 8)
+    parts = []
+    for r in range(3):
+        k = torch.empty(kw, dtype=torch.int64, device="cuda")
+        ctx.partial_device(T, m, k, r, 3, prec, 8)
+        parts.append(k)
+    merged = torch.stack(parts).min(dim=0).values
+    torch.cuda.synchronize()
+    assert torch.equal(merged, full)
