@@ -97,9 +97,26 @@ struct Plan {
     std::vector<double> cells;     // nb + 1 exclusive prefix of cells
 };
 
-Plan build_plan(int64_t d, int64_t n, int64_t excl, bool self, int prec, int64_t H) {
+// Tile height: a multiple of the re-seed interval H (re-seeds inside a tile happen at
+// warp-uniform steps, so taller tiles only amortise the per-tile stagger ramp), at most 4096
+// rows, and short enough to leave >= ~20k tiles for the persistent warps.
+#ifndef MP_TILE_MAX
+#define MP_TILE_MAX 4096
+#endif
+#ifndef MP_TILE_GROW_BELOW
+#define MP_TILE_GROW_BELOW 4096
+#endif
+int64_t tile_height(int64_t Hs, int64_t n, int64_t ndiag) {
+    int64_t H = Hs;
+    while (H < MP_TILE_GROW_BELOW && H * 2 <= MP_TILE_MAX && (double)ndiag * n / (H * 2) / 2.0 >= 20000.0) H *= 2;
+    return H;
+}
+
+Plan build_plan(int64_t d, int64_t n, int64_t excl, bool self, int prec, int64_t Hs) {
     Plan pl;
     pl.nc = mpk::pick_variant(prec, (int)d).NC;
+    const int64_t ndiag = self ? std::max<int64_t>(0, n - 1 - excl) : 2 * n - 1;
+    const int64_t H = tile_height(Hs, n, ndiag);
     pl.H = (int)H;
     if (self) { pl.dlo = excl + 1; pl.dhi = n - 1; }
     else { pl.dlo = -(n - 1); pl.dhi = n - 1; }
@@ -228,7 +245,7 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
             mp.t_begin = t_begin;
             mp.t_count = t_end - t_begin;
             mp.counter = (unsigned long long*)ctx->counter.p;
-            mp.n = n; mp.d = (int)d; mp.m = (int)m; mp.H = (int)H;
+            mp.n = n; mp.d = (int)d; mp.m = (int)m; mp.H = (int)H; mp.HT = pl.H;
             mp.delta_lo = pl.dlo; mp.delta_hi = pl.dhi;
             const int bps = std::max(1, mpk::main_blocks_per_sm(prec, (int)d, self));
             const long long want_warps = mp.t_count;

@@ -34,6 +34,12 @@
 #ifndef MP_MINB
 #define MP_MINB 1
 #endif
+#ifndef MP_MINB_F32
+#define MP_MINB_F32 3
+#endif
+#ifndef MP_KEEP_DL
+#define MP_KEEP_DL 16
+#endif
 
 namespace mpk {
 
@@ -245,7 +251,7 @@ template <int G, int W> struct Geo {
     static constexpr int NC = NL * W;                                    // cells (diagonals) per warp
     // ring positions move in batches of SB steps, prefetched one batch ahead: live rows
     // span CW(RA-1) + 2 SB, live columns 2 SB + CW - 1
-    static constexpr int SB = W == 1 ? 4 : 2;
+    static constexpr int SB = 4;
     static constexpr int RING_R = pow2ceil(CW * (RA - 1) + 2 * SB) < CW ? CW : pow2ceil(CW * (RA - 1) + 2 * SB);
     static constexpr int RPC = RING_R / CW;                              // ring rows per residue class
     static constexpr int RING_C = pow2ceil(2 * SB + CW - 1);
@@ -282,7 +288,7 @@ template <int DL, int G> __device__ __forceinline__ int rank_of_plane(int p) { r
 // minimum resident blocks per SM for the register budget (128 threads per block max)
 template <class T, int DL, int G, int W> constexpr int min_blocks() {
     // caps the register budget where ptxas still fits without spills (measured with -Xptxas -v)
-    return (sizeof(T) == 4 && G == 1 && DL * W <= 16) ? 3 : MP_MINB;
+    return (sizeof(T) == 4 && G == 1 && DL * W <= 16) ? MP_MINB_F32 : MP_MINB;
 }
 template <class T, int DL, int G, int W, bool SELF>
 __global__ void __launch_bounds__(128, (min_blocks<T, DL, G, W>()))
@@ -316,7 +322,7 @@ mp_diag(const MainParams p) {
     K* keys = reinterpret_cast<K*>(p.keys);
 
     const long long n = p.n;
-    const int d = p.d, m = p.m, H = p.H;
+    const int d = p.d, m = p.m, H = p.H, HT = p.HT;
     const T two_m = (T)(2 * m);
     const T INF = PT<T>::inf(), NINF = PT<T>::ninf();
 
@@ -436,8 +442,8 @@ mp_diag(const MainParams p) {
         const long long delta0 = p.delta_lo + b * Gm::NC;
         const long long delta1 = min(delta0 + Gm::NC - 1, p.delta_hi);
         const long long rlo = max(0ll, -delta1), rhi = min(n, n - max(delta0, 0ll));
-        const long long q = rlo / H + (t - __ldg(&p.seg_prefix[b]));
-        const long long r0 = max(q * H, rlo), r1 = min((q + 1) * H, rhi);
+        const long long q = rlo / HT + (t - __ldg(&p.seg_prefix[b]));
+        const long long r0 = max(q * HT, rlo), r1 = min((q + 1) * HT, rhi);
 
         // the lane's W cells: diagonals and valid row ranges inside the tile
         long long delta[W], lo[W], hi[W];
@@ -452,43 +458,42 @@ mp_diag(const MainParams p) {
 #pragma unroll
         for (int u = 0; u < W; ++u) { dlt[u] = (int)delta[u]; lo32[u] = (int)lo[u]; hi32[u] = (int)hi[u]; }
 
-        // seeds: direct centred dot products at row lo (reading G8),
-        // compensated (Kahan) accumulation.  Operands are position-major and padded to D
-        // dims, so a lane (G == 1) loads its DL dims of a window position as vectors.
+        // seeds: direct centred dot products (reading G8), compensated
+        // (Kahan) accumulation, at each cell's first row and then every H rows (reseed(),
+        // called at warp-uniform steps; the tile is HT >= H rows tall).  Operands are
+        // position-major and padded to D dims, so a lane (G == 1) loads its DL dims as vectors.
         T QT[W][DL];
-#pragma unroll
-        for (int u = 0; u < W; ++u) {
-            const bool ok = lo[u] < hi[u];
+        auto seed_cell = [&](int u, long long row) {
             T mq[DL], mr[DL], cmp[DL];
-            const long long i0 = ok ? lo[u] : 0, j0 = ok ? lo[u] + delta[u] : 0;
+            const long long i0 = row, j0 = row + delta[u];
             load_dims<T, DL, G>(mu_q + i0 * D, g, mq);
             load_dims<T, DL, G>(mu_r + j0 * D, g, mr);
 #pragma unroll
-            for (int kk = 0; kk < DL; ++kk) {
-                QT[u][kk] = (kk * G + g) >= d ? (T)-1 : (T)0;
-                cmp[kk] = (T)0;
-            }
-            if (ok) {
-                const T* xq_p = tw_q + i0 * D;
-                const T* xr_p = tw_r + j0 * D;
+            for (int kk = 0; kk < DL; ++kk) { QT[u][kk] = (T)0; cmp[kk] = (T)0; }
+            const T* xq_p = tw_q + i0 * D;
+            const T* xr_p = tw_r + j0 * D;
 #pragma unroll 2
-                for (int tt = 0; tt < m; ++tt) {
-                    T xq[DL], xr[DL];
-                    load_dims<T, DL, G>(xq_p + (long long)tt * D, g, xq);
-                    load_dims<T, DL, G>(xr_p + (long long)tt * D, g, xr);
+            for (int tt = 0; tt < m; ++tt) {
+                T xq[DL], xr[DL];
+                load_dims<T, DL, G>(xq_p + (long long)tt * D, g, xq);
+                load_dims<T, DL, G>(xr_p + (long long)tt * D, g, xr);
 #pragma unroll
-                    for (int kk = 0; kk < DL; ++kk) {
-                        const T y = (xq[kk] - mq[kk]) * (xr[kk] - mr[kk]) - cmp[kk];
-                        const T t2 = QT[u][kk] + y;
-                        cmp[kk] = (t2 - QT[u][kk]) - y;
-                        QT[u][kk] = t2;
-                    }
+                for (int kk = 0; kk < DL; ++kk) {
+                    const T y = (xq[kk] - mq[kk]) * (xr[kk] - mr[kk]) - cmp[kk];
+                    const T t2 = QT[u][kk] + y;
+                    cmp[kk] = (t2 - QT[u][kk]) - y;
+                    QT[u][kk] = t2;
                 }
-#pragma unroll
-                for (int kk = 0; kk < DL; ++kk)
-                    if ((kk * G + g) >= d) QT[u][kk] = (T)-1;  // padded dims (zero data)
             }
-        }
+#pragma unroll
+            for (int kk = 0; kk < DL; ++kk)
+                if ((kk * G + g) >= d) QT[u][kk] = (T)-1;  // padded dims (zero data)
+        };
+#pragma unroll
+        for (int u = 0; u < W; ++u)
+#pragma unroll
+            for (int kk = 0; kk < DL; ++kk) QT[u][kk] = (kk * G + g) >= d ? (T)-1 : (T)0;
+        int seeded_step = -1;  // step whose row was seeded at its batch start (re-seed)
 
         const int nrows = (int)(r1 - r0);
         const int s_end = nrows + CW * (RA - 1);
@@ -522,11 +527,15 @@ mp_diag(const MainParams p) {
                 active[u] = row >= lo32[u] && row < hi32[u];
                 upd[u] = row > lo32[u] && row < hi32[u];
             }
+            if (s == seeded_step) {  // QT of this row was just seeded
+#pragma unroll
+                for (int u = 0; u < W; ++u) upd[u] = false;
+            }
             const int scn = Gm::scol(col[W - 1]);
 
             // thresholds stay in registers for small per-lane dim counts; wide lanes
             // re-read them from the ring after the sort (register budget)
-            constexpr bool KEEP = (DL <= 16);
+            constexpr bool KEEP = (DL <= MP_KEEP_DL);
             T S[W][DL], tr[KEEP ? DL : 1], tc0[KEEP ? DL : 1];
 #pragma unroll
             for (int kk = 0; kk < DL; ++kk) {
@@ -664,6 +673,18 @@ mp_diag(const MainParams p) {
         };
 
         for (int s0 = 0; s0 < s_end; s0 += SB) {
+            // seeds: each cell's first row at s0 = 0, then the current row every H steps
+            // (H is a multiple of SB, so re-seeds fall on batch starts: one call site)
+            if (s0 % H == 0) {
+                const long long row = R0 + s0 - (long long)CW * a;
+#pragma unroll 1
+                for (int u = 0; u < W; ++u) {
+                    const bool first = s0 == 0;
+                    const long long sr_ = first ? lo[u] : row;
+                    if (first ? (lo[u] < hi[u]) : (row > lo[u] && row < hi[u])) seed_cell(u, sr_);
+                }
+                seeded_step = s0 == 0 ? -1 : s0;
+            }
             // evict positions no step from s0 on reads; prefetch the next batch's entries
             const int rx = min(max(s0 - CW * (RA - 1), 0), nrows);
             evict(true, R0, row_out, rx);
@@ -678,7 +699,7 @@ mp_diag(const MainParams p) {
             col_in = max(col_in, c_need);
             cp_async_commit();
             if constexpr (W == 2) {  // ping-pong the carried column registers (no moves)
-#pragma unroll
+#pragma unroll 1
                 for (int k2 = 0; k2 < SB; k2 += 2) {
                     if (s0 + k2 < s_end) step(s0 + k2, carA, carB);
                     if (s0 + k2 + 1 < s_end) step(s0 + k2 + 1, carB, carA);

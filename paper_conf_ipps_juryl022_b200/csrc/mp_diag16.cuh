@@ -68,7 +68,7 @@ mp_diag_h(const MainParams p) {
     unsigned long long* keys = reinterpret_cast<unsigned long long*>(p.keys);
 
     const long long n = p.n;
-    const int d = p.d, m = p.m, H = p.H;
+    const int d = p.d, m = p.m, H = p.H, HT = p.HT;
     const int n32 = (int)n;
     const __half2 two_m = __float2half2_rn((float)(2 * m));
     const float FINF = __int_as_float(0x7f800000);
@@ -187,8 +187,8 @@ mp_diag_h(const MainParams p) {
         const long long delta0 = p.delta_lo + b * Gm::NC;
         const long long delta1 = min(delta0 + Gm::NC - 1, p.delta_hi);
         const long long rlo = max(0ll, -delta1), rhi = min(n, n - max(delta0, 0ll));
-        const long long q = rlo / H + (t - __ldg(&p.seg_prefix[b]));
-        const long long r0 = max(q * H, rlo), r1 = min((q + 1) * H, rhi);
+        const long long q = rlo / HT + (t - __ldg(&p.seg_prefix[b]));
+        const long long r0 = max(q * HT, rlo), r1 = min((q + 1) * HT, rhi);
 
         long long delta[2], lo[2], hi[2];
         int dlt[2], lo32[2], hi32[2];
@@ -203,15 +203,14 @@ mp_diag_h(const MainParams p) {
 
         // seeds at each cell's first row: Mixed -> FP32 operands and compensated FP32
         // accumulation rounded to half (FP32 precalc); FP16 -> half arithmetic throughout
-        // seeds at the pair's first row (both cells start at row r0 except at diagonal starts):
+        // seeds (at the pair's first rows, then every H rows at warp-uniform steps):
         // Mixed -> FP32 operands and FP32 accumulation rounded to half (the FP32 precalc);
         // FP16 -> half arithmetic.  The row window is shared by the pair and the second cell's
         // column window is the first one shifted by one position.
         __half2 QT[DL];
-        {
+        auto seed_pair = [&](bool ok0, bool ok1, long long row0, long long row1) {
             using TA = typename std::conditional<MIXED, float, __half>::type;
-            const bool ok0 = lo[0] < hi[0], ok1 = lo[1] < hi[1];
-            const bool same = ok0 && ok1 && lo[0] == lo[1];
+            const bool same = ok0 && ok1 && row0 == row1;
             TA acc0[DL], acc1[DL];
 #pragma unroll
             for (int kk = 0; kk < DL; ++kk) { acc0[kk] = (TA)0.f; acc1[kk] = (TA)0.f; }
@@ -219,7 +218,7 @@ mp_diag_h(const MainParams p) {
             for (int u = 0; u < (same ? 1 : 2); ++u) {
                 const bool ok = u == 0 ? ok0 : ok1;
                 if (!ok) continue;
-                const long long i0 = lo[u], j0 = lo[u] + delta[u];
+                const long long i0 = u == 0 ? row0 : row1, j0 = i0 + delta[u];
                 TA mq[DL], mr0[DL], mr1[DL];
 #pragma unroll
                 for (int kk = 0; kk < DL; ++kk) {
@@ -236,26 +235,29 @@ mp_diag_h(const MainParams p) {
                     for (int kk = 0; kk < DL; ++kk) {
                         const TA xq = tw_q[(i0 + tt) * D + kk * G + g];
                         const TA xr = xr_prev[kk];
+                        const TA xn = tw_r[(j0 + tt + 1) * D + kk * G + g];
                         if (same) {
-                            const TA xn = tw_r[(j0 + tt + 1) * D + kk * G + g];
                             acc0[kk] = acc0[kk] + (xq - mq[kk]) * (xr - mr0[kk]);
                             acc1[kk] = acc1[kk] + (xq - mq[kk]) * (xn - mr1[kk]);
-                            xr_prev[kk] = xn;
                         } else {
                             TA& acc = u == 0 ? acc0[kk] : acc1[kk];
                             acc = acc + (xq - mq[kk]) * (xr - mr0[kk]);
-                            xr_prev[kk] = tw_r[(j0 + tt + 1) * D + kk * G + g];
                         }
+                        xr_prev[kk] = xn;
                     }
                 }
             }
 #pragma unroll
             for (int kk = 0; kk < DL; ++kk) {
                 const bool pad = (kk * G + g) >= d;
-                const float v0 = pad ? -1.f : (float)acc0[kk], v1 = pad ? -1.f : (float)acc1[kk];
-                QT[kk] = __floats2half2_rn(v0, v1);
+                const __half h0 = __float2half_rn(pad ? -1.f : (float)acc0[kk]);
+                const __half h1 = __float2half_rn(pad ? -1.f : (float)acc1[kk]);
+                QT[kk] = __halves2half2(ok0 ? h0 : __low2half(QT[kk]), ok1 ? h1 : __high2half(QT[kk]));
             }
-        }
+        };
+#pragma unroll
+        for (int kk = 0; kk < DL; ++kk) QT[kk] = __float2half2_rn((kk * G + g) >= d ? -1.f : 0.f);
+        int seeded_step = -1;
 
         const int nrows = (int)(r1 - r0);
         const int s_end = nrows + CW * (RA - 1);
@@ -284,6 +286,7 @@ mp_diag_h(const MainParams p) {
                 active[u] = row >= lo32[u] && row < hi32[u];
                 upd[u] = row > lo32[u] && row < hi32[u];
             }
+            if (s == seeded_step) upd[0] = upd[1] = false;  // QT of this row was just seeded
             __half2 S[DL], tr[DL], tc[DL];
             if (upd[0] == upd[1]) {
 #pragma unroll
@@ -396,6 +399,16 @@ mp_diag_h(const MainParams p) {
         };
 
         for (int s0 = 0; s0 < s_end; s0 += SB) {
+            if (s0 % H == 0) {  // seeds: first rows at s0 = 0, current row every H steps
+                const long long row = R0 + s0 - (long long)CW * a;
+                if (s0 == 0) {
+                    seed_pair(lo[0] < hi[0], lo[1] < hi[1], lo[0], lo[1]);
+                } else {
+                    const bool u0 = row > lo[0] && row < hi[0], u1 = row > lo[1] && row < hi[1];
+                    if (u0 || u1) seed_pair(u0, u1, row, row);
+                }
+                seeded_step = s0 == 0 ? -1 : s0;
+            }
             const int rx = min(max(s0 - CW * (RA - 1), 0), nrows);
             evict(true, R0, row_out, rx);
             row_out = rx;

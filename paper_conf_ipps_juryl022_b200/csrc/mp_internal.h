@@ -20,7 +20,8 @@ struct MainParams {
     long long t_begin, t_count;   // tile range of this launch
     unsigned long long* counter;  // zeroed before launch
     long long n;                  // subsequences
-    int d, m, H;                  // dims, window, re-seed interval (tile height)
+    int d, m, H;                  // dims, window, re-seed interval H (rows)
+    int HT;                       // tile height (multiple of H)
     long long delta_lo, delta_hi; // diagonal range [lo, hi] (j = i + delta)
 };
 

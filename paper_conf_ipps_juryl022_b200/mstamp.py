@@ -16,7 +16,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "lib", "libmstamp_b200.so")
+LIB_PATH = os.environ.get("MP_LIB_PATH") or os.path.join(_HERE, "lib", "libmstamp_b200.so")
 
 PRECISIONS = {"fp64": 0, "fp32": 1, "fp16": 2, "mixed": 3}
 STATUS = {0: "MP_OK", 1: "MP_ERR_INVALID", 2: "MP_ERR_NOMEM", 3: "MP_ERR_CUDA", 4: "MP_ERR_NCCL",

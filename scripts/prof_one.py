@@ -7,7 +7,12 @@ import torch  # noqa: E402
 
 from paper_conf_ipps_juryl022_b200 import datagen, mstamp  # noqa: E402
 
-cfg = datagen.make(sys.argv[1] if len(sys.argv) > 1 else "C2")
+name = sys.argv[1] if len(sys.argv) > 1 else "C2"
+if name.startswith("X"):   # X<d>_<n>_<m>: ad-hoc self-join shape for profiling, e.g. X64_32768_256
+    d_, n_, m_ = (int(v) for v in name[1:].split("_"))
+    cfg = dict(T=datagen.random_walk(d_, n_, m_, 7), Tr=None, d=d_, n=n_, m=m_, exclusion=m_ // 4)
+else:
+    cfg = datagen.make(name)
 prec = sys.argv[2] if len(sys.argv) > 2 else "fp32"
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
 d, n, m, e = cfg["d"], cfg["n"], cfg["m"], cfg["exclusion"]
