@@ -2,6 +2,7 @@
 // The fused diagonal kernel itself lives in mp_diag.cuh (instantiated in inst_*.cu so
 // the heavy template variants compile in parallel).
 #include "mp_diag16.cuh"
+#include "mp_diag64f.cuh"
 
 namespace mpk {
 
@@ -297,8 +298,8 @@ Variant pick_variant(int prec, int d) {
         else if (dp <= 256) { v.DL = 8; v.G = dp / 8; }
         else { v.DL = dp / 32; v.G = 32; }
         v.W = 2;
-    } else if (prec == P64) {
-        if (dp <= 16) { v.DL = dp; v.G = 1; v.W = dp <= 8 ? 2 : 1; }
+    } else if (prec == P64) {  // FP64 with the FP32 filter (mp_diag64f): one cell per lane-cell
+        if (dp <= 16) { v.DL = dp; v.G = 1; v.W = 1; }
         else { v.DL = 16; v.G = dp / 16; v.W = 1; }
     } else {
         if (dp <= 8) { v.DL = dp; v.G = 1; v.W = 2; }
@@ -323,9 +324,6 @@ static long long dispatch_t(int op, int DL, int G, int W, const MainParams* p, i
     if constexpr (sizeof(T) == 4) {
         MP_CASE(1, 1, 2) MP_CASE(2, 1, 2) MP_CASE(4, 1, 2) MP_CASE(8, 1, 2) MP_CASE(16, 1, 1)
         MP_CASE(16, 2, 1) MP_CASE(16, 4, 1) MP_CASE(16, 8, 1) MP_CASE(16, 16, 1) MP_CASE(16, 32, 1) MP_CASE(32, 32, 1)
-    } else {
-        MP_CASE(1, 1, 2) MP_CASE(2, 1, 2) MP_CASE(4, 1, 2) MP_CASE(8, 1, 2) MP_CASE(16, 1, 1)
-        MP_CASE(16, 2, 1) MP_CASE(16, 4, 1) MP_CASE(16, 8, 1) MP_CASE(16, 16, 1) MP_CASE(16, 32, 1)
     }
 #undef MP_CASE
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
@@ -346,11 +344,26 @@ static long long dispatch_h(int op, int DL, int G, const MainParams* p, int grid
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
 }
 
+template <bool SELF>
+static long long dispatch_64f(int op, int DL, int G, const MainParams* p, int grid, cudaStream_t s) {
+#define MP_FCASE(dl, g)                                                                    \
+    if (DL == dl && G == g) {                                                              \
+        if (op == 0) return (long long)Inst64F<dl, g, SELF>::smem();                       \
+        if (op == 1) return (long long)Inst64F<dl, g, SELF>::launch(*p, grid, s);          \
+        if (op == 3) return Inst64F<dl, g, SELF>::warps_per_block();                       \
+        return Inst64F<dl, g, SELF>::blocks_per_sm();                                      \
+    }
+    MP_FCASE(1, 1) MP_FCASE(2, 1) MP_FCASE(4, 1) MP_FCASE(8, 1) MP_FCASE(16, 1)
+    MP_FCASE(16, 2) MP_FCASE(16, 4) MP_FCASE(16, 8) MP_FCASE(16, 16) MP_FCASE(16, 32)
+#undef MP_FCASE
+    return op == 1 ? (long long)cudaErrorInvalidValue : 0;
+}
+
 static long long dispatch(int op, int prec, bool self, int d, const MainParams* p, int grid, cudaStream_t s) {
     const Variant v = pick_variant(prec, d);
     if (prec == P16) return self ? dispatch_h<true, false>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, false>(op, v.DL, v.G, p, grid, s);
     if (prec == PMIX) return self ? dispatch_h<true, true>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, true>(op, v.DL, v.G, p, grid, s);
-    if (prec == P64) return self ? dispatch_t<double, true>(op, v.DL, v.G, v.W, p, grid, s) : dispatch_t<double, false>(op, v.DL, v.G, v.W, p, grid, s);
+    if (prec == P64) return self ? dispatch_64f<true>(op, v.DL, v.G, p, grid, s) : dispatch_64f<false>(op, v.DL, v.G, p, grid, s);
     if (prec == P32) return self ? dispatch_t<float, true>(op, v.DL, v.G, v.W, p, grid, s) : dispatch_t<float, false>(op, v.DL, v.G, v.W, p, grid, s);
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
 }
