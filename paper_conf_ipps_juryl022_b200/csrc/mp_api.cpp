@@ -204,7 +204,7 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     for (int sidx = 0; sidx < (self ? 1 : 2); ++sidx) {
         Buf** B = series_bufs[sidx];
         MP_CUDA(ctx, ensure(*B[0], (size_t)n * d * sb));
-        if (half) MP_CUDA(ctx, ensure(*B[1], (size_t)n * d * sb));
+        if (half) MP_CUDA(ctx, ensure(*B[1], (size_t)(n + 1) * d * sb));  // pair format: n+1 entries
         MP_CUDA(ctx, ensure(*B[2], (size_t)n * d * tb));
         MP_CUDA(ctx, ensure(*B[3], (size_t)n * Dp * tb));
         MP_CUDA(ctx, ensure(*B[4], (size_t)L * Dp * tb));

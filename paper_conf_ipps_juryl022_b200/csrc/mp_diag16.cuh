@@ -98,12 +98,12 @@ mp_diag_h(const MainParams p) {
         for (int e = lane; e < cnt * D; e += 32) {
             const int pi = e / D, pl = e - pi * D;
             const int pos = base + p_lo + pi;
-            if (pos < 0 || pos >= n32) continue;
+            if (pos < (is_row ? 0 : -1) || pos >= n32) continue;   // column pair -1 = (none, col 0)
             const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
             if (pl == 0) dflag[sl] = 0;
             H4* dst = &buf[pl * ps + sl];
             if (pl < d) {
-                const H4* src = st + (size_t)pos * d + pl;
+                const H4* src = st + (size_t)(is_row ? pos : pos + 1) * d + pl;
                 cp_async8(dst, src);
                 cp_async4(&dst->z, &src->z);
             } else {  // padded dimension: a = +inf with QT = -1 gives D = +inf
@@ -112,7 +112,7 @@ mp_diag_h(const MainParams p) {
                 dst->z = __half2half2(HINF);
             }
             const int rk = rank_of_plane<DL, G>(pl);
-            if (rk < d && want_thr) {
+            if (rk < d && want_thr && pos >= 0) {
                 const unsigned long long* kp = keys + (size_t)pos * d + rk;
                 cp_async4(&bb[pl * ps + sl], reinterpret_cast<const char*>(kp) + 4);
                 cp_async4(&ib[pl * ps + sl], kp);
@@ -133,7 +133,7 @@ mp_diag_h(const MainParams p) {
         for (int e = lane; e < cnt * D; e += 32) {
             const int pi = e / D, pl = e - pi * D;
             const int pos = base + p_lo + pi;
-            if (pos < 0 || pos >= n32) continue;
+            if (pos < (is_row ? 0 : -1) || pos >= n32) continue;
             if (is_row) {
                 const int sl = Gm::srow(pos);
                 buf[pl * ps + sl].w = __half2half2(__float2half_rn(bb[pl * ps + sl]));

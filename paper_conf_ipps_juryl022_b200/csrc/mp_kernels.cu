@@ -188,26 +188,33 @@ __global__ void pre_diff_h(const PreParams p) {
     flat[n * d + o] = __float2half_rn(dg);
     flat[2 * n * d + o] = __float2half_rn(av);
 }
-// row format (x, x) and pair format (x_pos, x_pos+1) H4 entries for the half2 kernel
+// row format (x, x) and pair format (x_pos, x_pos+1) H4 entries for the half2 kernel.  The
+// pair array has n+1 entries: entry e holds (x_{e-1}, x_e), so a pair starting at column -1
+// (an AB-join diagonal start) still finds its second cell's data.
 __global__ void pre_fmt_h(const PreParams p) {
     const long long n = p.n;
     const int d = p.d;
     const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-    if (gid >= n * d) return;
-    const long long pos = gid / d;
+    if (gid >= (n + 1) * d) return;
+    const long long e = gid / d;          // pair entry; first position e - 1
+    const int dim = (int)(gid % d);
     const __half* f = reinterpret_cast<const __half*>(p.flat);
     const long long nd = n * d;
     const __half z = __float2half(0.f);
-    H4 r, q;
-    r.x = __half2half2(f[gid]); r.y = __half2half2(f[nd + gid]); r.z = __half2half2(f[2 * nd + gid]);
-    r.w = __half2half2(z);
-    const bool nx = pos + 1 < n;
-    q.x = __halves2half2(f[gid], nx ? f[gid + d] : z);
-    q.y = __halves2half2(f[nd + gid], nx ? f[nd + gid + d] : z);
-    q.z = __halves2half2(f[2 * nd + gid], nx ? f[2 * nd + gid + d] : z);
+    const long long ia = (e - 1) * d + dim, ib = e * d + dim;
+    const bool va = e >= 1, vb = e < n;
+    H4 q;
+    q.x = __halves2half2(va ? f[ia] : z, vb ? f[ib] : z);
+    q.y = __halves2half2(va ? f[nd + ia] : z, vb ? f[nd + ib] : z);
+    q.z = __halves2half2(va ? f[2 * nd + ia] : z, vb ? f[2 * nd + ib] : z);
     q.w = __half2half2(z);
-    reinterpret_cast<H4*>(p.st)[gid] = r;
     reinterpret_cast<H4*>(p.st_pair)[gid] = q;
+    if (vb) {
+        H4 r;
+        r.x = __half2half2(f[ib]); r.y = __half2half2(f[nd + ib]); r.z = __half2half2(f[2 * nd + ib]);
+        r.w = __half2half2(z);
+        reinterpret_cast<H4*>(p.st)[ib] = r;
+    }
 }
 template <class T>
 __global__ void pre_pm_h(const PreParams p) {
@@ -400,7 +407,7 @@ cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s) {
             pre_diff_h<__half><<<grid1d(cnt, 256), 256, 0, s>>>(p);
             pre_pm_h<__half><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
         }
-        pre_fmt_h<<<grid1d(cnt, 256), 256, 0, s>>>(p);
+        pre_fmt_h<<<grid1d((p.n + 1) * p.d, 256), 256, 0, s>>>(p);
     }
     return cudaGetLastError();
 }

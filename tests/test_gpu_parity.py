@@ -236,6 +236,15 @@ def test_half_modes_ab_and_bands(ctx, prec):
     Tq, Tr = datagen.random_walk_ab(d, n, m, 54)
     Pg, Ig = ctx.compute(Tq, m, prec, Tr=Tr)
     assert np.all(np.isfinite(Pg)) and np.all((Ig >= 0) & (Ig < n))
+    # error vs the GPU FP64 result (itself oracle-checked) stays within the stated bound; an
+    # AB-join exercises the diagonal starts at column 0 (pairs beginning at column -1)
+    P64, I64 = ctx.compute(Tq, m, "fp64", Tr=Tr)
+    st = _half_stats(P64, I64, Pg, Ig, m)
+    print(prec, "ab", st)
+    assert st["median_rel"] < (0.02 if prec == "mixed" else 0.2)
+    a, b = datagen.motif_positions(n, m)
+    for k in range(d // 2):
+        assert Ig[k, a] == b
     T = torch.from_numpy(datagen.random_walk(d, n, m, 55)).cuda()
     kw = mstamp.key_words(d, n, prec)
     full = torch.empty(kw, dtype=torch.int64, device="cuda")
