@@ -490,10 +490,15 @@ mp_diag(const MainParams p) {
                 if ((kk * G + g) >= d) QT[u][kk] = (T)-1;  // padded dims (zero data)
         };
 #pragma unroll
-        for (int u = 0; u < W; ++u)
+        for (int u = 0; u < W; ++u) {
+            if (lo[u] < hi[u]) {
+                seed_cell(u, lo[u]);
+            } else {
 #pragma unroll
-            for (int kk = 0; kk < DL; ++kk) QT[u][kk] = (kk * G + g) >= d ? (T)-1 : (T)0;
-        int seeded_step = -1;  // step whose row was seeded at its batch start (re-seed)
+                for (int kk = 0; kk < DL; ++kk) QT[u][kk] = (kk * G + g) >= d ? (T)-1 : (T)0;
+            }
+        }
+        int seeded_step = -1;  // step whose row was re-seeded at its batch start
 
         const int nrows = (int)(r1 - r0);
         const int s_end = nrows + CW * (RA - 1);
@@ -675,15 +680,12 @@ mp_diag(const MainParams p) {
         for (int s0 = 0; s0 < s_end; s0 += SB) {
             // seeds: each cell's first row at s0 = 0, then the current row every H steps
             // (H is a multiple of SB, so re-seeds fall on batch starts: one call site)
-            if (s0 % H == 0) {
+            if (s0 > 0 && s0 % H == 0) {
                 const long long row = R0 + s0 - (long long)CW * a;
 #pragma unroll 1
-                for (int u = 0; u < W; ++u) {
-                    const bool first = s0 == 0;
-                    const long long sr_ = first ? lo[u] : row;
-                    if (first ? (lo[u] < hi[u]) : (row > lo[u] && row < hi[u])) seed_cell(u, sr_);
-                }
-                seeded_step = s0 == 0 ? -1 : s0;
+                for (int u = 0; u < W; ++u)
+                    if (row > lo[u] && row < hi[u]) seed_cell(u, row);
+                seeded_step = s0;
             }
             // evict positions no step from s0 on reads; prefetch the next batch's entries
             const int rx = min(max(s0 - CW * (RA - 1), 0), nrows);

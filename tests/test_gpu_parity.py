@@ -257,3 +257,25 @@ def test_half_modes_ab_and_bands(ctx, prec):
     merged = torch.stack(parts).min(dim=0).values
     torch.cuda.synchronize()
     assert torch.equal(merged, full)
+
+
+@pytest.mark.parametrize("prec", ["fp32", "mixed"])
+def test_c3_sampled_rows(ctx, oracle_mod, prec):
+    """BASELINE config C3 at full size (self-join d=64, n=262144, m=256: the sort/scan-dominated
+    regime, lane groups of G lanes per cell); sampled rows against the oracle (FP32: the 1e-4
+    gate; Mixed: the stated error bound) plus properties at every (k, i)."""
+    cfg = datagen.make("C3")
+    T, m, e, n = cfg["T"], cfg["m"], cfg["exclusion"], cfg["n"]
+    Pg, Ig = ctx.compute(T, m, prec, e)
+    a, b = datagen.motif_positions(n, m)
+    rows = np.unique(np.concatenate([[0, n - 1, a, b], np.random.default_rng(6).integers(0, n, 4)]))
+    P, I, P2 = oracle_mod.mstamp(T, m, e, rows=rows)
+    if prec == "fp32":
+        st = parity.check(oracle_mod, T, m, P, I, P2, Pg, Ig, prec, rows=rows)
+    else:
+        st = _half_stats(P, I, Pg[:, rows], Ig[:, rows], m)
+        assert st["median_rel"] < 0.02
+    print(prec, st)
+    for k in range(32):
+        assert Ig[k, a] == b and Ig[k, b] == a
+    assert np.all(np.diff(Pg, axis=0) >= -1e-3 * Pg[1:])
