@@ -226,6 +226,8 @@ def main():
     ap.add_argument("--ref-seconds", type=float, default=15.0)
     ap.add_argument("--no-per-precision", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--backend", default="nccl", help="process-group backend for N>1 (gloo: functional "
+                    "test of the multi-rank path, e.g. several ranks on one GPU via MP_BENCH_DEVICE)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
@@ -237,10 +239,13 @@ def main():
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = int(os.environ.get("MP_BENCH_DEVICE", os.environ.get("LOCAL_RANK", "0")))
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(args.backend)
     dev = torch.device("cuda", local)
     cfg = datagen.make(args.config)
     d, n, m, e = cfg["d"], cfg["n"], cfg["m"], cfg["exclusion"]
@@ -326,16 +331,20 @@ def main():
     if rank == 0:
         peaks, src = load_peaks()
         cells = computed_cells(n, e, self_join)
+        # roofline of the dominant kernel: algorithmic ops of the cells THIS launch computed (rank
+        # 0's band when N > 1) over its CUDA-event duration
+        band_cells = cells
         if world > 1:
-            cells = cells  # each rank's kernel time is for its band; report job-level ops / max time
-        ops = alu_ops_per_cell_dim(d, self_join) * cells * d
+            _, bc = mstamp.plan_bands(d, n, m, args.precision, e, self_join, world)
+            band_cells = int(bc[0])
+        ops = alu_ops_per_cell_dim(d, self_join) * band_cells * d
         peak_tops = SM_COUNT * ALU_LANES * NOMINAL_SM_MHZ * 1e6 / 1e12
         achieved = ops / (kms * 1e-3) / 1e12 if kms > 0 else None
         roof = {"bound": "alu", "achieved": achieved, "peak": peak_tops, "unit": "Tops/s",
                 "frac": achieved / peak_tops if achieved else None,
                 "traffic": load_traffic(args.config, args.precision),
                 "kernel": "mp_diag", "ops_per_cell_dim": alu_ops_per_cell_dim(d, self_join),
-                "computed_cell_dims": cells * d,
+                "computed_cell_dims": band_cells * d,
                 "peak_basis": f"148 SM x 64 ALU lanes/clk x {NOMINAL_SM_MHZ:.0f} MHz (derived; MEASURED_PEAKS {src} "
                               "has no ALU figure)"}
         cpu = None
