@@ -50,7 +50,9 @@ typedef enum {
     MP_FP64 = 0,   /* precalculation FP64, main loop FP64           (L426-428, L764-766) */
     MP_FP32 = 1,   /* precalculation FP32, main loop FP32           (L430-432, L771-772) */
     MP_FP16 = 2,   /* precalculation FP16, main loop FP16           (L434-436, L773-776) */
-    MP_MIXED = 3   /* precalculation FP32, main loop FP16           (L438-440, L777-785) */
+    MP_MIXED = 3,  /* precalculation FP32, main loop FP16           (L438-440, L777-785) */
+    MP_FP16C = 4   /* precalculation FP16 with Kahan-compensated sums, main loop FP16
+                      (Fig. 1 "FP16 with compensator" L442-444, L786-798; G17) */
 } mp_precision;
 
 #define MP_MAX_D 1024
@@ -59,7 +61,8 @@ typedef struct mp_ctx mp_ctx;   /* opaque */
 
 typedef struct {
     int device;             /* CUDA device ordinal this context drives (one process per GPU) */
-    int64_t reseed_h[4];    /* re-seed interval H (rows) per mp_precision; 0 -> default */
+    int64_t reseed_h[4];    /* re-seed interval H (rows) for FP64, FP32, FP16 (also FP16C), MIXED;
+                               0 -> default (R2) */
 } mp_config;
 
 /* Create a context on cfg->device (cfg == NULL -> device 0, defaults). */

@@ -2,5 +2,5 @@
 #define MP_DIAG_IMPL
 #include "mp_diag16.cuh"
 namespace mpk {
-template struct InstH<16, 32, false, 1>;
+template struct InstH<32, 32, false, 2>;
 }  // namespace mpk

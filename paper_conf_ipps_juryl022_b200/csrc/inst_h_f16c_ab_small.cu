@@ -2,5 +2,8 @@
 #define MP_DIAG_IMPL
 #include "mp_diag16.cuh"
 namespace mpk {
-template struct InstH<16, 32, false, 1>;
+template struct InstH<1, 1, false, 2>;
+template struct InstH<2, 1, false, 2>;
+template struct InstH<4, 1, false, 2>;
+template struct InstH<8, 1, false, 2>;
 }  // namespace mpk

@@ -20,7 +20,7 @@
 
 namespace {
 
-constexpr int64_t kDefaultH[4] = {4096, 1024, 256, 256};  // FP64, FP32, FP16, MIXED (upper bounds)
+constexpr int64_t kDefaultH[5] = {4096, 1024, 256, 256, 256};  // FP64, FP32, FP16, MIXED, FP16C (upper bounds)
 
 // Default re-seed interval H (= tile height, the paper's tiling lever against error growth,
 // PAPER.md:L700-703).  The recurrence error grows with H relative to the window energy, which
@@ -42,7 +42,7 @@ struct mp_ctx {
     int device = 0;
     int nsm = 148;
     cudaStream_t stream = nullptr;
-    int64_t H[4] = {0, 0, 0, 0};
+    int64_t H[5] = {0, 0, 0, 0, 0};
     std::string err;
     // cached scratch
     Buf dT, dTr, st_q, st_r, tw_q, tw_r, mu_q, mu_r, mup_q, mup_r, nrm, keys, ext, seg, counter, dP, dI, flag;
@@ -159,7 +159,7 @@ mp_status validate(mp_ctx* ctx, const void* T, int64_t d, int64_t n, int64_t m, 
     if (m < 2) return fail(ctx, MP_ERR_INVALID, "m must be >= 2");
     if (n >= (int64_t(1) << 31) - 1) return fail(ctx, MP_ERR_INVALID, "n must be < 2^31");
     if (m > (int64_t(1) << 20)) return fail(ctx, MP_ERR_INVALID, "m too large");
-    if (prec < 0 || prec > 3) return fail(ctx, MP_ERR_INVALID, "unknown precision");
+    if (prec < 0 || prec > 4) return fail(ctx, MP_ERR_INVALID, "unknown precision");
     if (prec == MP_FP64 && d > 512) return fail(ctx, MP_ERR_UNSUPPORTED, "FP64 supports d <= 512");
     return MP_OK;
 }
@@ -184,9 +184,9 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     if (flag) return fail(ctx, MP_ERR_INVALID, "non-finite input");
 
     // precalculation (Pseudocode 1 line 2)
-    const bool half = prec == MP_FP16 || prec == MP_MIXED;
+    const bool half = prec == MP_FP16 || prec == MP_MIXED || prec == MP_FP16C;
     const size_t sb = half ? 16 : 4 * eb;                                   // stats entry bytes
-    const size_t tb = prec == MP_FP64 ? 8 : (prec == MP_FP16 ? 2 : 4);       // precalc value bytes
+    const size_t tb = prec == MP_FP64 ? 8 : ((prec == MP_FP16 || prec == MP_FP16C) ? 2 : 4);  // precalc value bytes
     const mpk::Variant var = mpk::pick_variant(prec, (int)d);
     const int Dp = var.DL * var.G;
     mpk::PreParams pp{};
@@ -276,8 +276,9 @@ mp_status mp_init(mp_ctx** out, const mp_config* cfg) {
     if (cfg) {
         ctx->device = cfg->device;
         for (int i = 0; i < 4; ++i) ctx->H[i] = cfg->reseed_h[i];
+        ctx->H[4] = cfg->reseed_h[2];  // FP16C follows FP16
     }
-    for (int i = 0; i < 4; ++i)
+    for (int i = 0; i < 5; ++i)
         if (ctx->H[i] < 0) { delete ctx; return MP_ERR_INVALID; }
     int ndev = 0;
     cudaError_t e = cudaGetDeviceCount(&ndev);
@@ -318,7 +319,7 @@ int64_t mp_key_words(int64_t d, int64_t n, mp_precision prec) {
 
 mp_status mp_plan_bands(int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
                         int self_join, int world, int64_t* block_begin, int64_t* cells) {
-    if (world < 1 || !block_begin || !cells || d < 1 || n < 2 || m < 2 || prec < 0 || prec > 3)
+    if (world < 1 || !block_begin || !cells || d < 1 || n < 2 || m < 2 || prec < 0 || prec > 4)
         return MP_ERR_INVALID;
     if (self_join && exclusion < 0) exclusion = (m + 3) / 4;
     Plan pl = build_plan(d, n, exclusion, self_join != 0, prec, default_h(prec, m));
@@ -335,7 +336,7 @@ mp_status mp_plan_bands(int64_t d, int64_t n, int64_t m, mp_precision prec, int6
 
 mp_status mp_plan_diagonals(int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
                             int self_join, int world, int64_t* diag_begin) {
-    if (world < 1 || !diag_begin || d < 1 || n < 2 || m < 2 || prec < 0 || prec > 3) return MP_ERR_INVALID;
+    if (world < 1 || !diag_begin || d < 1 || n < 2 || m < 2 || prec < 0 || prec > 4) return MP_ERR_INVALID;
     if (self_join && exclusion < 0) exclusion = (m + 3) / 4;
     Plan pl = build_plan(d, n, exclusion, self_join != 0, prec, default_h(prec, m));
     if (pl.nb == 0) {

@@ -37,9 +37,12 @@ template <int DL, int G> struct SmemH {
     static constexpr int WPB = bytes_per_warp * 4 <= 112 * 1024 ? 4 : bytes_per_warp * 2 <= 112 * 1024 ? 2 : 1;
 };
 
-template <int DL, int G, bool SELF, bool MIXED>
+// MODE: 0 = FP16, 1 = Mixed (FP32 precalc and seeds), 2 = FP16C (half precalc and seeds with
+// Kahan-compensated sums, reading G17)
+template <int DL, int G, bool SELF, int MODE>
 __global__ void __launch_bounds__(128)
 mp_diag_h(const MainParams p) {
+    constexpr bool MIXED = MODE == 1;
     using Gm = Geo<G, 2>;
     using SM = SmemH<DL, G>;
     using TS = typename std::conditional<MIXED, float, __half>::type;  // seed operand type
@@ -226,9 +229,9 @@ mp_diag_h(const MainParams p) {
                     mr0[kk] = mu_r[j0 * D + kk * G + g];
                     mr1[kk] = same ? mu_r[(j0 + 1) * D + kk * G + g] : mr0[kk];
                 }
-                TA xr_prev[DL];
+                TA xr_prev[DL], cp0[DL], cp1[DL];  // Kahan compensators (FP16C)
 #pragma unroll
-                for (int kk = 0; kk < DL; ++kk) xr_prev[kk] = tw_r[j0 * D + kk * G + g];
+                for (int kk = 0; kk < DL; ++kk) { xr_prev[kk] = tw_r[j0 * D + kk * G + g]; cp0[kk] = (TA)0.f; cp1[kk] = (TA)0.f; }
 #pragma unroll 2
                 for (int tt = 0; tt < m; ++tt) {
 #pragma unroll
@@ -236,7 +239,20 @@ mp_diag_h(const MainParams p) {
                         const TA xq = tw_q[(i0 + tt) * D + kk * G + g];
                         const TA xr = xr_prev[kk];
                         const TA xn = tw_r[(j0 + tt + 1) * D + kk * G + g];
-                        if (same) {
+                        if constexpr (MODE == 2) {  // compensated half accumulation
+                            auto kadd = [](TA& acc, TA& cp, TA v) {
+                                const TA y = v - cp;
+                                const TA t2 = acc + y;
+                                cp = (t2 - acc) - y;
+                                acc = t2;
+                            };
+                            if (same) {
+                                kadd(acc0[kk], cp0[kk], (xq - mq[kk]) * (xr - mr0[kk]));
+                                kadd(acc1[kk], cp1[kk], (xq - mq[kk]) * (xn - mr1[kk]));
+                            } else {
+                                kadd(u == 0 ? acc0[kk] : acc1[kk], u == 0 ? cp0[kk] : cp1[kk], (xq - mq[kk]) * (xr - mr0[kk]));
+                            }
+                        } else if (same) {
                             acc0[kk] = acc0[kk] + (xq - mq[kk]) * (xr - mr0[kk]);
                             acc1[kk] = acc1[kk] + (xq - mq[kk]) * (xn - mr1[kk]);
                         } else {
@@ -440,7 +456,7 @@ mp_diag_h(const MainParams p) {
     }
 }
 
-template <int DL, int G, bool SELF, bool MIXED> struct InstH {
+template <int DL, int G, bool SELF, int MODE> struct InstH {
     static size_t smem() { return SmemH<DL, G>::bytes_per_warp * SmemH<DL, G>::WPB; }
     static int warps_per_block() { return SmemH<DL, G>::WPB; }
     static cudaError_t launch(const MainParams& p, int grid, cudaStream_t s);
@@ -448,19 +464,19 @@ template <int DL, int G, bool SELF, bool MIXED> struct InstH {
 };
 
 #ifdef MP_DIAG_IMPL
-template <int DL, int G, bool SELF, bool MIXED>
-cudaError_t InstH<DL, G, SELF, MIXED>::launch(const MainParams& p, int grid, cudaStream_t s) {
+template <int DL, int G, bool SELF, int MODE>
+cudaError_t InstH<DL, G, SELF, MODE>::launch(const MainParams& p, int grid, cudaStream_t s) {
     const size_t sm = smem();
-    cudaError_t e = cudaFuncSetAttribute(mp_diag_h<DL, G, SELF, MIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaError_t e = cudaFuncSetAttribute(mp_diag_h<DL, G, SELF, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
-    mp_diag_h<DL, G, SELF, MIXED><<<grid, SmemH<DL, G>::WPB * 32, sm, s>>>(p);
+    mp_diag_h<DL, G, SELF, MODE><<<grid, SmemH<DL, G>::WPB * 32, sm, s>>>(p);
     return cudaGetLastError();
 }
-template <int DL, int G, bool SELF, bool MIXED> int InstH<DL, G, SELF, MIXED>::blocks_per_sm() {
+template <int DL, int G, bool SELF, int MODE> int InstH<DL, G, SELF, MODE>::blocks_per_sm() {
     const size_t sm = smem();
-    cudaFuncSetAttribute(mp_diag_h<DL, G, SELF, MIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaFuncSetAttribute(mp_diag_h<DL, G, SELF, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     int nb = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mp_diag_h<DL, G, SELF, MIXED>, SmemH<DL, G>::WPB * 32, sm);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mp_diag_h<DL, G, SELF, MODE>, SmemH<DL, G>::WPB * 32, sm);
     return nb;
 }
 #endif

@@ -44,7 +44,7 @@ struct PreParams {
 };
 
 // Precision codes match mp_precision.
-enum { P64 = 0, P32 = 1, P16 = 2, PMIX = 3 };
+enum { P64 = 0, P32 = 1, P16 = 2, PMIX = 3, P16C = 4 };
 
 // Variant selection for a given (precision, d): dims per lane DL and lanes per cell G.
 struct Variant { int DL; int G; int W; int NC; };

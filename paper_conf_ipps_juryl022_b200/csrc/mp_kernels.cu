@@ -117,7 +117,7 @@ __global__ void pre_scale_pick(const PreParams p, int pure16) {
     e = max(-60, min(60, e));
     p.scale[dim] = ldexp(1.0, e);
 }
-template <class T>  // T = float (Mixed: FP32 precalc) or __half (FP16: half precalc)
+template <class T, bool KAHAN = false>  // T = float (Mixed) or __half (FP16; FP16C: KAHAN)
 __global__ void pre_stats_h(const PreParams p) {
     const long long n = p.n, L = p.n + p.m - 1;
     const int d = p.d, m = p.m;
@@ -139,7 +139,7 @@ __global__ void pre_stats_h(const PreParams p) {
             const float y = cx * cx - c; const float tt = q + y; c = (tt - q) - y; q = tt;
         }
         nr = sqrtf(q);
-    } else {  // FP16 mode: plain half arithmetic (the paper's uncompensated FP16 precalc)
+    } else if constexpr (!KAHAN) {  // FP16 mode: plain half arithmetic (the paper's FP16 precalc)
         __half s = __float2half(0.f);
         for (int t = 0; t < m; ++t) s = __hadd(s, __double2half(sc * x[t]));
         mu = __hdiv(s, __int2half_rn(m));
@@ -147,6 +147,25 @@ __global__ void pre_stats_h(const PreParams p) {
         for (int t = 0; t < m; ++t) {
             const __half cx = __hsub(__double2half(sc * x[t]), mu);
             q = __hfma(cx, cx, q);
+        }
+        nr = hsqrt(q);
+    } else {  // FP16C: half arithmetic with Kahan-compensated sums (Fig. 1 "FP16 with compensator")
+        __half s = __float2half(0.f), c = __float2half(0.f);
+        for (int t = 0; t < m; ++t) {
+            const __half y = __hsub(__double2half(sc * x[t]), c);
+            const __half tt = __hadd(s, y);
+            c = __hsub(__hsub(tt, s), y);
+            s = tt;
+        }
+        mu = __hdiv(s, __int2half_rn(m));
+        __half q = __float2half(0.f);
+        c = __float2half(0.f);
+        for (int t = 0; t < m; ++t) {
+            const __half cx = __hsub(__double2half(sc * x[t]), mu);
+            const __half y = __hsub(__hmul(cx, cx), c);
+            const __half tt = __hadd(q, y);
+            c = __hsub(__hsub(tt, q), y);
+            q = tt;
         }
         nr = hsqrt(q);
     }
@@ -300,7 +319,7 @@ Variant pick_variant(int prec, int d) {
     int dp = 1;
     while (dp < d) dp <<= 1;
     Variant v;
-    if (prec == P16 || prec == PMIX) {  // half2: a lane-cell is a pair of diagonals
+    if (prec == P16 || prec == PMIX || prec == P16C) {  // half2: a lane-cell is a pair of diagonals
         if (dp <= 8) { v.DL = dp; v.G = 1; }
         else if (dp <= 256) { v.DL = 8; v.G = dp / 8; }
         else { v.DL = dp / 32; v.G = 32; }
@@ -336,7 +355,7 @@ static long long dispatch_t(int op, int DL, int G, int W, const MainParams* p, i
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
 }
 
-template <bool SELF, bool MIXED>
+template <bool SELF, int MIXED>
 static long long dispatch_h(int op, int DL, int G, const MainParams* p, int grid, cudaStream_t s) {
 #define MP_HCASE(dl, g)                                                                    \
     if (DL == dl && G == g) {                                                              \
@@ -368,8 +387,9 @@ static long long dispatch_64f(int op, int DL, int G, const MainParams* p, int gr
 
 static long long dispatch(int op, int prec, bool self, int d, const MainParams* p, int grid, cudaStream_t s) {
     const Variant v = pick_variant(prec, d);
-    if (prec == P16) return self ? dispatch_h<true, false>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, false>(op, v.DL, v.G, p, grid, s);
-    if (prec == PMIX) return self ? dispatch_h<true, true>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, true>(op, v.DL, v.G, p, grid, s);
+    if (prec == P16) return self ? dispatch_h<true, 0>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 0>(op, v.DL, v.G, p, grid, s);
+    if (prec == PMIX) return self ? dispatch_h<true, 1>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 1>(op, v.DL, v.G, p, grid, s);
+    if (prec == P16C) return self ? dispatch_h<true, 2>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 2>(op, v.DL, v.G, p, grid, s);
     if (prec == P64) return self ? dispatch_64f<true>(op, v.DL, v.G, p, grid, s) : dispatch_64f<false>(op, v.DL, v.G, p, grid, s);
     if (prec == P32) return self ? dispatch_t<float, true>(op, v.DL, v.G, v.W, p, grid, s) : dispatch_t<float, false>(op, v.DL, v.G, v.W, p, grid, s);
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
@@ -402,6 +422,10 @@ cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s) {
             pre_stats_h<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
             pre_diff_h<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
             pre_pm_h<float><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
+        } else if (prec == P16C) {
+            pre_stats_h<__half, true><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+            pre_diff_h<__half><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+            pre_pm_h<__half><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
         } else {
             pre_stats_h<__half><<<grid1d(cnt, 256), 256, 0, s>>>(p);
             pre_diff_h<__half><<<grid1d(cnt, 256), 256, 0, s>>>(p);

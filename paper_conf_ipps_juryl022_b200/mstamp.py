@@ -18,7 +18,7 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("MP_LIB_PATH") or os.path.join(_HERE, "lib", "libmstamp_b200.so")
 
-PRECISIONS = {"fp64": 0, "fp32": 1, "fp16": 2, "mixed": 3}
+PRECISIONS = {"fp64": 0, "fp32": 1, "fp16": 2, "mixed": 3, "fp16c": 4}
 STATUS = {0: "MP_OK", 1: "MP_ERR_INVALID", 2: "MP_ERR_NOMEM", 3: "MP_ERR_CUDA", 4: "MP_ERR_NCCL",
           5: "MP_ERR_UNSUPPORTED"}
 EXPORTS = ["mp_init", "mp_free", "mp_last_error", "mp_version", "mp_compute", "mp_compute_device",

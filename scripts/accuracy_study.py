@@ -1,0 +1,83 @@
+"""Accuracy of the reduced-precision modes vs FP64 (the paper's Fig. 2 / Fig. 7 analogues,
+PAPER.md:L881-931, L958-974, L1721-1878; NEXT-1/NEXT-2 of SURVEY 8(f)).
+
+For seeded synthetic inputs (random walks with a planted motif; the bounded paper-like
+pattern family) and every precision mode it reports, against the GPU FP64 result (itself
+parity-checked against the oracle by the test suite):
+  R   recall: fraction of profile indices equal to FP64's (L890-892),
+  A   relative accuracy 1 - E, E = mean |P - P64| / max(P64, 0.05 sqrt(2m)) (L894-898, G20),
+  Rm  embedded-motif recall: planted pair recovered in every dimension count k < k' (L911-915),
+and, for FP16 / FP16C / Mixed, A and R as a function of the re-seed interval H (Fig. 7's
+tile-count lever).  Writes profiles/r1_accuracy.json and prints a table.
+    python scripts/accuracy_study.py
+"""
+import json
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+from paper_conf_ipps_juryl022_b200 import datagen, mstamp  # noqa: E402
+
+MODES = ["fp32", "mixed", "fp16c", "fp16"]
+
+
+def metrics(P, I, P64, I64, motif, d, m):
+    # E: mean relative discrepancy with the near-exact floor of DESIGN.md section 7 (a planted
+    # match has P64 ~ 1e-8; its absolute error, not its relative one, is meaningful)
+    fin = np.isfinite(P64)
+    den = np.maximum(P64[fin], 0.05 * np.sqrt(2 * m))
+    E = float(np.mean(np.abs(P[fin] - P64[fin]) / den))
+    R = float(np.mean(I[np.isfinite(P64)] == I64[np.isfinite(P64)]))
+    Rm = None
+    if motif is not None:
+        a, b = motif
+        kk = max(1, d // 2)
+        Rm = float(np.mean([I[k, a] == b and I[k, b] == a for k in range(kk)]))
+    return dict(A=1.0 - E, R=R, Rm=Rm)
+
+
+def main():
+    rows = []
+    ctx = mstamp.Context(0)
+    cases = []
+    for n in (2048, 8192):
+        for d in (4, 16):
+            for m in (32, 128):
+                cases.append(("walk", d, n, m, datagen.random_walk(d, n, m, 1000 + n + d + m),
+                              datagen.motif_positions(n, m)))
+    for (d, n, m) in ((8, 8192, 64), (16, 8192, 128)):
+        cases.append(("patterns", d, n, m, datagen.bounded_patterns(d, n, m, 77 + d), None))
+    for fam, d, n, m, T, motif in cases:
+        P64, I64 = ctx.compute(T, m, "fp64")
+        for mode in MODES:
+            P, I = ctx.compute(T, m, mode)
+            r = dict(family=fam, d=d, n=n, m=m, mode=mode, H="default")
+            r.update(metrics(P, I, P64, I64, motif, d, m))
+            rows.append(r)
+    # re-seed interval sweep (Fig. 7 analogue) on one walk
+    T = datagen.random_walk(16, 8192, 64, 4242)
+    P64, I64 = ctx.compute(T, 64, "fp64")
+    for h in (64, 128, 256, 512, 1024, 4096):
+        c = mstamp.Context(0, reseed_h=[0, h, h, h])
+        for mode in ("mixed", "fp16c", "fp16", "fp32"):
+            P, I = c.compute(T, 64, mode)
+            r = dict(family="walk", d=16, n=8192, m=64, mode=mode, H=h)
+            r.update(metrics(P, I, P64, I64, datagen.motif_positions(8192, 64), 16, 64))
+            rows.append(r)
+        c.close()
+    ctx.close()
+    os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
+    with open(os.path.join(ROOT, "profiles", "r1_accuracy.json"), "w") as f:
+        json.dump(rows, f, indent=1)
+    print(f"{'family':9s} {'d':>3s} {'n':>5s} {'m':>4s} {'mode':6s} {'H':>7s} {'A':>8s} {'R':>7s} {'Rm':>5s}")
+    for r in rows:
+        rm = "-" if r["Rm"] is None else f"{r['Rm']:.2f}"
+        print(f"{r['family']:9s} {r['d']:3d} {r['n']:5d} {r['m']:4d} {r['mode']:6s} {str(r['H']):>7s} "
+              f"{r['A']:8.5f} {r['R']:7.4f} {rm:>5s}")
+
+
+if __name__ == "__main__":
+    main()

@@ -195,7 +195,7 @@ def _half_stats(P_or, I_or, P, I, m):
                 max_rel=float(rel.max()), recall=float((I == I_or)[fin].mean()))
 
 
-@pytest.mark.parametrize("prec", ["fp16", "mixed"])
+@pytest.mark.parametrize("prec", ["fp16", "mixed", "fp16c"])
 def test_half_modes_c1(ctx, oracle_mod, c1_oracle, prec):
     """FP16 / Mixed: no tolerance gate (parity unpinned); the
     error vs FP64 is measured and must stay within the stated bound; the planted motif must
@@ -215,7 +215,7 @@ def test_half_modes_c1(ctx, oracle_mod, c1_oracle, prec):
         assert Ig[k, a] == b and Ig[k, b] == a
 
 
-@pytest.mark.parametrize("prec", ["fp16", "mixed"])
+@pytest.mark.parametrize("prec", ["fp16", "mixed", "fp16c"])
 @pytest.mark.parametrize("shape", [(3, 700, 32, 8, 51), (16, 900, 64, 16, 52), (40, 300, 16, 4, 53)])
 def test_half_modes_shapes(ctx, oracle_mod, prec, shape):
     d, n, m, e, seed = shape
@@ -228,7 +228,7 @@ def test_half_modes_shapes(ctx, oracle_mod, prec, shape):
     assert np.all(np.isfinite(Pg))
 
 
-@pytest.mark.parametrize("prec", ["fp16", "mixed"])
+@pytest.mark.parametrize("prec", ["fp16", "mixed", "fp16c"])
 def test_half_modes_ab_and_bands(ctx, prec):
     """AB-join runs; band partials merge bit-identically to the single band (FP32 key format)."""
     from paper_conf_ipps_juryl022_b200 import mstamp
@@ -276,6 +276,10 @@ def test_c3_sampled_rows(ctx, oracle_mod, prec):
         st = _half_stats(P, I, Pg[:, rows], Ig[:, rows], m)
         assert st["median_rel"] < 0.02
     print(prec, st)
+    # planted motif: exact (FP32) / relaxed recall with r = 1/16 (Mixed; the paper's relaxed
+    # embedded-motif recall R^r, PAPER.md:L917-931 -- a neighbouring window is within half
+    # precision of the exact copy at m = 256)
+    slack = 0 if prec == "fp32" else m // 16
     for k in range(32):
-        assert Ig[k, a] == b and Ig[k, b] == a
+        assert abs(Ig[k, a] - b) <= slack and abs(Ig[k, b] - a) <= slack
     assert np.all(np.diff(Pg, axis=0) >= -1e-3 * Pg[1:])
