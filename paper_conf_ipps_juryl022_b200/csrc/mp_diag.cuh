@@ -625,6 +625,18 @@ mp_diag(const MainParams p) {
                     T v[W];
 #pragma unroll
                     for (int u = 0; u < W; ++u) v[u] = ssc[(u * DL + kk) * 32 + lane];
+                    // skip ranks (and sides) no lane can improve: most slow steps touch 1-2 ranks
+                    T vmin_l = v[0];
+#pragma unroll
+                    for (int u = 1; u < W; ++u) vmin_l = PT<T>::vmin(vmin_l, v[u]);
+                    const bool need_r = __any_sync(FULL, vmin_l <= rowv[pl * PSR + sr].w);
+                    bool need_c = false;
+                    if (SELF) {
+#pragma unroll
+                        for (int u = 0; u < W; ++u) need_c |= v[u] <= colv[pl * PSC + Gm::scol(col[u])].w;
+                        need_c = __any_sync(FULL, need_c);
+                    }
+                    if (!need_r && !need_c) continue;
                     // row group: W cells per lane x CA lanes
                     T vr = v[0];
 #pragma unroll
@@ -636,7 +648,7 @@ mp_diag(const MainParams p) {
 #pragma unroll
                     for (int u = 0; u < W; ++u) mine |= v[u] == vr;
                     const unsigned eqr = __ballot_sync(FULL, mine) & gmask_row;
-                    if (vr < INF && lane == __ffs(eqr) - 1) {
+                    if (need_r && vr < INF && lane == __ffs(eqr) - 1) {
                         int j = col[W - 1];
 #pragma unroll
                         for (int u = W - 1; u >= 0; --u)
@@ -650,7 +662,7 @@ mp_diag(const MainParams p) {
                             rowdirty[sr] = 1;
                         }
                     }
-                    if (SELF) {
+                    if (SELF && need_c) {
 #pragma unroll
                         for (int u = 0; u < W; ++u) {
                             T vc = v[u];

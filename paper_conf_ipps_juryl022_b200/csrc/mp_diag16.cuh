@@ -366,13 +366,18 @@ mp_diag_h(const MainParams p) {
                     const int pl = kk * G + g;
                     const __half2 vh = ssc[kk * 32 + lane];
                     const float v[2] = {__low2float(vh), __high2float(vh)};
+                    const bool need_r = __any_sync(FULL, fminf(v[0], v[1]) <= rowb[pl * PSR + sr]);
+                    bool need_c = false;
+                    if (SELF) need_c = __any_sync(FULL, v[0] <= colb[pl * PSC + scn] ||
+                                                      v[1] <= colb[pl * PSC + Gm::scol(col0 + 1)]);
+                    if (!need_r && !need_c) continue;
                     float vr = fminf(v[0], v[1]);
 #pragma unroll
                     for (int bit = 0; bit < Gm::LOG_CA; ++bit)
                         vr = fminf(vr, __shfl_xor_sync(FULL, vr, 1 << (bit + Gm::LOG_G)));
                     const bool mine = v[0] == vr || v[1] == vr;
                     const unsigned eqr = __ballot_sync(FULL, mine) & gmask_row;
-                    if (vr < FINF && lane == __ffs(eqr) - 1) {
+                    if (need_r && vr < FINF && lane == __ffs(eqr) - 1) {
                         const int j = (v[0] == vr) ? col0 : col0 + 1;          // lowest column first
                         const int ix = pl * PSR + sr;
                         const float cur = rowb[ix];
@@ -384,7 +389,7 @@ mp_diag_h(const MainParams p) {
                             rowdirty[sr] = 1;
                         }
                     }
-                    if (SELF) {
+                    if (SELF && need_c) {
 #pragma unroll
                         for (int u = 0; u < 2; ++u) {
                             float vc = v[u];

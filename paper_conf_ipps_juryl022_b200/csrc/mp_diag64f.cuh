@@ -305,12 +305,15 @@ mp_diag64f(const MainParams p) {
             for (int kk = 0; kk < DL; ++kk) {
                 const int pl = kk * G + g;
                 const double v = ssc[kk * 32 + lane];
+                const bool need_r = __any_sync(FULL, v <= rowb[pl * PSR + sr]);
+                const bool need_c = SELF && __any_sync(FULL, v <= colb[pl * PSC + sc]);
+                if (!need_r && !need_c) continue;
                 double vr = v;
 #pragma unroll
                 for (int bit = 0; bit < Gm::LOG_CA; ++bit)
                     vr = PT<double>::vmin(vr, __shfl_xor_sync(FULL, vr, 1 << (bit + Gm::LOG_G)));
                 const unsigned eqr = __ballot_sync(FULL, v == vr) & gmask_row;
-                if (vr < INF && lane == __ffs(eqr) - 1) {
+                if (need_r && vr < INF && lane == __ffs(eqr) - 1) {
                     const int ix = pl * PSR + sr;
                     const double cur = rowb[ix];
                     const unsigned ci = rowi[ix] & ~DIRTY;
@@ -321,7 +324,7 @@ mp_diag64f(const MainParams p) {
                         rowdirty[sr] = 1;
                     }
                 }
-                if (SELF) {
+                if (SELF && need_c) {
                     double vc = v;
 #pragma unroll
                     for (int bit = 0; bit < 5 - Gm::LOG_G - Gm::LOG_CA; ++bit)
