@@ -37,6 +37,11 @@
 #ifndef MP_MINB_F32
 #define MP_MINB_F32 3
 #endif
+#ifndef MP_W1_UNROLL
+#define MP_W1_UNROLL 1
+#endif
+#define MP_PRAGMA(x) _Pragma(#x)
+#define MP_UNROLL(n) MP_PRAGMA(unroll n)
 #ifndef MP_KEEP_DL
 #define MP_KEEP_DL 16
 #endif
@@ -720,7 +725,7 @@ mp_diag(const MainParams p) {
                 }
             } else {  // one copy of the step body (instruction-cache footprint)
                 const int s1 = min(s0 + SB, s_end);
-#pragma unroll 1
+                MP_UNROLL(MP_W1_UNROLL)
                 for (int ss = s0; ss < s1; ++ss) step(ss, carA, carB);
             }
             cp_async_wait_all();   // this lane's prefetch for the next batch has landed

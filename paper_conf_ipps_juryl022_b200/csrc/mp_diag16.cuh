@@ -1,20 +1,24 @@
 #pragma once
-// mp_diag16.cuh -- the fused diagonal kernel in half precision (FP16 and Mixed modes,
-// PAPER.md Fig. 1 table L420-444, Sec. III-C L773-785: "FP16 for storage and computation";
-// Mixed differs only in a FP32 precalculation, done by the precompute kernels).
+// mp_diag16.cuh -- the fused diagonal kernel in half precision (FP16, Mixed and FP16C modes,
+// PAPER.md Fig. 1 table L420-444, Sec. III-C L773-790: "FP16 for storage and computation";
+// Mixed differs in a FP32 precalculation, FP16C in compensated half sums).
 //
 // Same structure as mp_diag (mp_diag.cuh): warp tiles of consecutive diagonals, staggered
 // lane-cells, per-warp shared-memory rings staged by cp.async one batch ahead, filtered
-// min/argmin with a warp-shuffle slow path and packed-key merges.  Differences:
+// min/argmin with a warp-shuffle slow path.  Differences:
 //   * a lane-cell is a PAIR of adjacent diagonals (delta, delta+1) packed into __half2, so
 //     every FMA / min / max / compare of the main loop processes two cells (HFMA2, HMNMX2);
-//   * row ring entries hold duplicated half2 (x, x); column ring entries hold the pair
+//   * row ring entries are 8 B (df, dg, a, threshold as halves; the .H0_H0 operand swizzle
+//     broadcasts them to both cells for free); column ring entries hold the pair
 //     (x_c, x_{c+1}) (precomputed in global memory), so one LDS.128 feeds both cells;
-//   * the authoritative running best per (position, rank) is an FP32 value (exact: it is a
-//     half converted to float) + index in separate arrays; the half2 thresholds in the ring
-//     are filter copies refreshed after staging and on updates.
+//   * every running best is a half value, so the ring's half threshold IS the best: the slow
+//     path compares against it and writes improvements straight through to the global merge
+//     key (RED.MIN.64 on (float bits << 32 | j), which also applies the lowest-index tie
+//     rule); there is no eviction pass.  Thresholds enter the ring through a 4 B float
+//     staging slot (cp.async of the key's value word) converted once the copy has landed.
 // Keys, finalize and the multi-GPU merge are the FP32 ones (float bits << 32 | j).
 #include <cuda_fp16.h>
+#include <type_traits>
 #include "mp_diag.cuh"
 
 namespace mpk {
@@ -24,18 +28,50 @@ template <> struct PT<__half2> {
     static __device__ __forceinline__ __half2 vmax(__half2 a, __half2 b) { return __hmax2(a, b); }
 };
 
-struct alignas(16) H4 { __half2 x, y, z, w; };  // (df, dg, a, threshold) for a cell pair
+struct alignas(8) RH { __half df, dg, a, t; };   // row ring entry (one position)
+struct alignas(16) H4 { __half2 x, y, z, w; };   // column ring entry (pair c, c+1)
+
+// warps per block (1..4) that maximise resident warps per SM under the shared-memory budget
+// (228 KB per SM, 1 KB reserved per block, 227 KB per block, 32 blocks per SM)
+constexpr int best_wpb(size_t bpw) {
+    int best = 1, bw = 0;
+    for (int w = 1; w <= 4; ++w) {
+        if (bpw * w > 227u * 1024u) break;
+        int nb = (int)((228u * 1024u) / (bpw * w + 1024u));
+        if (nb > 32) nb = 32;
+        if (nb * w >= bw) { bw = nb * w; best = w; }
+    }
+    return best;
+}
 
 template <int DL, int G> struct SmemH {
     using Gm = Geo<G, 2>;
     static constexpr int D = DL * G;
-    // rings: H4 entries + authoritative best (float value, u32 index) per (plane, slot)
-    static constexpr size_t ring_bytes =
-        (((size_t)D * (Gm::PSR + Gm::PSC) * (sizeof(H4) + 8)) + 15) & ~(size_t)15;
-    static constexpr size_t flag_bytes = ((Gm::RING_R + Gm::RING_C) * 4 + 15) & ~(size_t)15;
-    static constexpr size_t bytes_per_warp = ring_bytes + flag_bytes + (size_t)DL * 32 * sizeof(__half2);
-    static constexpr int WPB = bytes_per_warp * 4 <= 112 * 1024 ? 4 : bytes_per_warp * 2 <= 112 * 1024 ? 2 : 1;
+    static constexpr size_t a16(size_t x) { return (x + 15) & ~(size_t)15; }
+    static constexpr size_t col_bytes = (size_t)D * Gm::PSC * sizeof(H4);
+    static constexpr size_t row_bytes = a16((size_t)D * Gm::PSR * sizeof(RH));
+    static constexpr size_t thr_bytes = a16((size_t)D * (Gm::PSR + Gm::PSC) * sizeof(float));
+    static constexpr size_t bytes_per_warp = col_bytes + row_bytes + thr_bytes + (size_t)DL * 32 * sizeof(__half2);
+    static constexpr int WPB = best_wpb(bytes_per_warp);
 };
+
+// DL operands of plane kk*G + g from a position-major row (vector loads when G == 1)
+template <class T, int DL, int G>
+__device__ __forceinline__ void ldv(const T* __restrict__ rowp, int g, T (&out)[DL]) {
+    constexpr int PER = 16 / (int)sizeof(T);
+    if constexpr (G == 1 && DL % PER == 0) {
+#pragma unroll
+        for (int q = 0; q < DL / PER; ++q) {
+            const uint4 v = __ldg(reinterpret_cast<const uint4*>(rowp) + q);
+            const T* e = reinterpret_cast<const T*>(&v);
+#pragma unroll
+            for (int r = 0; r < PER; ++r) out[q * PER + r] = e[r];
+        }
+    } else {
+#pragma unroll
+        for (int kk = 0; kk < DL; ++kk) out[kk] = rowp[kk * G + g];
+    }
+}
 
 // MODE: 0 = FP16, 1 = Mixed (FP32 precalc and seeds), 2 = FP16C (half precalc and seeds with
 // Kahan-compensated sums, reading G17)
@@ -52,17 +88,13 @@ mp_diag_h(const MainParams p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     unsigned char* wbase = smem_raw + (size_t)warp * SM::bytes_per_warp;
-    H4* rowv = reinterpret_cast<H4*>(wbase);
-    H4* colv = rowv + (size_t)D * PSR;
-    float* rowb = reinterpret_cast<float*>(colv + (size_t)D * PSC);
+    H4* colv = reinterpret_cast<H4*>(wbase);
+    RH* rowv = reinterpret_cast<RH*>(wbase + SM::col_bytes);
+    float* rowb = reinterpret_cast<float*>(wbase + SM::col_bytes + SM::row_bytes);
     float* colb = rowb + (size_t)D * PSR;
-    unsigned* rowi = reinterpret_cast<unsigned*>(colb + (size_t)D * PSC);
-    unsigned* coli = rowi + (size_t)D * PSR;
-    unsigned* rowdirty = reinterpret_cast<unsigned*>(wbase + SM::ring_bytes);
-    unsigned* coldirty = rowdirty + Gm::RING_R;
-    __half2* ssc = reinterpret_cast<__half2*>(wbase + SM::ring_bytes + SM::flag_bytes);
+    __half2* ssc = reinterpret_cast<__half2*>(wbase + SM::col_bytes + SM::row_bytes + SM::thr_bytes);
 
-    const H4* __restrict__ st_q = reinterpret_cast<const H4*>(p.st_q);   // row format (x, x)
+    const RH* __restrict__ st_q = reinterpret_cast<const RH*>(p.st_q);   // row format
     const H4* __restrict__ st_r = reinterpret_cast<const H4*>(p.st_r);   // pair format (x_c, x_c+1)
     const TS* __restrict__ tw_q = reinterpret_cast<const TS*>(p.tw_q);
     const TS* __restrict__ tw_r = reinterpret_cast<const TS*>(p.tw_r);
@@ -75,7 +107,7 @@ mp_diag_h(const MainParams p) {
     const int n32 = (int)n;
     const __half2 two_m = __float2half2_rn((float)(2 * m));
     const float FINF = __int_as_float(0x7f800000);
-    const __half HINF = __ushort_as_half(0x7c00), HNINF = __ushort_as_half(0xfc00);
+    const __half HZERO = __float2half(0.f), HINF = __ushort_as_half(0x7c00);
 
     const int lc = lane >> Gm::LOG_G, g = lane & (G - 1);
     const int a = lc >> Gm::LOG_CA, c = lc & (CA - 1);
@@ -85,93 +117,62 @@ mp_diag_h(const MainParams p) {
 #pragma unroll
     for (int aa = 0; aa < RA; ++aa) gmask_col |= 1u << (((aa * CA + c) << Gm::LOG_G) + g);
 
-    // ---- staging: stats by cp.async (12 B of the 16 B entry), authoritative best from the
-    // merge key (value half -> float, index half -> u32); the half2 filter copies of the
-    // thresholds are written by fixup() once the copies have landed.
+    // ---- staging: stats by cp.async, the key's value word into the float staging slot;
+    // fixup() writes the half thresholds once the copies have landed.  Column pairs start
+    // at position -1 (the pair (-1, 0) feeds cells whose first column is 0).
     auto stage = [&](bool is_row, int base, int p_lo, int p_hi) {
         const int cnt = p_hi - p_lo;
         if (cnt <= 0) return;
-        H4* buf = is_row ? rowv : colv;
         float* bb = is_row ? rowb : colb;
-        unsigned* ib = is_row ? rowi : coli;
-        unsigned* dflag = is_row ? rowdirty : coldirty;
         const int ps = is_row ? PSR : PSC;
-        const H4* __restrict__ st = is_row ? st_q : st_r;
         const bool want_thr = is_row || SELF;
         for (int e = lane; e < cnt * D; e += 32) {
             const int pi = e / D, pl = e - pi * D;
             const int pos = base + p_lo + pi;
-            if (pos < (is_row ? 0 : -1) || pos >= n32) continue;   // column pair -1 = (none, col 0)
+            if (pos < (is_row ? 0 : -1) || pos >= n32) continue;
             const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
-            if (pl == 0) dflag[sl] = 0;
-            H4* dst = &buf[pl * ps + sl];
-            if (pl < d) {
-                const H4* src = st + (size_t)(is_row ? pos : pos + 1) * d + pl;
-                cp_async8(dst, src);
-                cp_async4(&dst->z, &src->z);
-            } else {  // padded dimension: a = +inf with QT = -1 gives D = +inf
-                dst->x = __half2half2(__float2half(0.f));
-                dst->y = dst->x;
-                dst->z = __half2half2(HINF);
+            if (is_row) {
+                RH* dst = &rowv[pl * PSR + sl];
+                if (pl < d) {
+                    cp_async8(dst, st_q + (size_t)pos * d + pl);        // (df, dg, a, -)
+                } else {  // padded dimension: a = +inf with QT = -1 gives D = +inf
+                    dst->df = HZERO; dst->dg = HZERO; dst->a = HINF;
+                }
+            } else {
+                H4* dst = &colv[pl * PSC + sl];
+                if (pl < d) {
+                    const H4* src = st_r + (size_t)(pos + 1) * d + pl;
+                    cp_async8(dst, src);
+                    cp_async4(&dst->z, &src->z);
+                } else {
+                    dst->x = __half2half2(HZERO); dst->y = dst->x; dst->z = __half2half2(HINF);
+                }
             }
             const int rk = rank_of_plane<DL, G>(pl);
-            if (rk < d && want_thr && pos >= 0) {
-                const unsigned long long* kp = keys + (size_t)pos * d + rk;
-                cp_async4(&bb[pl * ps + sl], reinterpret_cast<const char*>(kp) + 4);
-                cp_async4(&ib[pl * ps + sl], kp);
-            } else {
-                bb[pl * ps + sl] = -FINF;
-                ib[pl * ps + sl] = 0x7fffffffu;
-            }
+            if (rk < d && want_thr && pos >= 0)
+                cp_async4(&bb[pl * ps + sl], reinterpret_cast<const char*>(keys + (size_t)pos * d + rk) + 4);
+            else
+                bb[pl * ps + sl] = -FINF;  // never hit
         }
     };
-    // thresholds (half) from the landed authoritative bests: row (t, t); column c -> low half
-    // of slot c and high half of slot c-1 (the pair (c-1, c))
+    // half thresholds from the landed values (exact: every stored best is a half value):
+    // row -> .t; column c -> low half of slot c and high half of slot c-1 (the pair (c-1, c))
     auto fixup = [&](bool is_row, int base, int p_lo, int p_hi) {
         const int cnt = p_hi - p_lo;
         if (cnt <= 0) return;
-        H4* buf = is_row ? rowv : colv;
-        const float* bb = is_row ? rowb : colb;
-        const int ps = is_row ? PSR : PSC;
         for (int e = lane; e < cnt * D; e += 32) {
             const int pi = e / D, pl = e - pi * D;
             const int pos = base + p_lo + pi;
             if (pos < (is_row ? 0 : -1) || pos >= n32) continue;
             if (is_row) {
-                const int sl = Gm::srow(pos);
-                buf[pl * ps + sl].w = __half2half2(__float2half_rn(bb[pl * ps + sl]));
+                const int ix = pl * PSR + Gm::srow(pos);
+                rowv[ix].t = __float2half_rn(rowb[ix]);
             } else {
-                const int sl = Gm::scol(pos);
-                const __half h = __float2half_rn(bb[pl * ps + sl]);
-                reinterpret_cast<__half*>(&buf[pl * ps + sl].w)[0] = h;
-                reinterpret_cast<__half*>(&buf[pl * ps + Gm::scol(pos - 1)].w)[1] = h;
+                const int ix = pl * PSC + Gm::scol(pos);
+                const __half h = __float2half_rn(colb[ix]);
+                reinterpret_cast<__half*>(&colv[ix].w)[0] = h;
+                if (pos >= 0) reinterpret_cast<__half*>(&colv[pl * PSC + Gm::scol(pos - 1)].w)[1] = h;
             }
-        }
-    };
-    auto evict = [&](bool is_row, int base, int p_lo, int p_hi) {
-        if (!is_row && !SELF) return;
-        const int cnt = p_hi - p_lo;
-        if (cnt <= 0) return;
-        const float* bb = is_row ? rowb : colb;
-        const unsigned* ib = is_row ? rowi : coli;
-        const unsigned* dflag = is_row ? rowdirty : coldirty;
-        const int ps = is_row ? PSR : PSC;
-        bool any = false;
-        for (int pi = lane; pi < cnt; pi += 32) {
-            const int pos = base + p_lo + pi;
-            if (pos >= 0 && pos < n32) any |= dflag[is_row ? Gm::srow(pos) : Gm::scol(pos)] != 0;
-        }
-        if (!__any_sync(FULL, any)) return;
-        for (int e = lane; e < cnt * D; e += 32) {
-            const int pi = e / D, pl = e - pi * D;
-            const int pos = base + p_lo + pi;
-            if (pos < 0 || pos >= n32) continue;
-            const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
-            if (dflag[sl] == 0) continue;
-            const int rk = rank_of_plane<DL, G>(pl);
-            if (rk >= d) continue;
-            const unsigned ix = ib[pl * ps + sl];
-            if (ix & DIRTY) KeyOps<float>::merge(keys + (size_t)pos * d + rk, bb[pl * ps + sl], ix & ~DIRTY);
         }
     };
 
@@ -204,63 +205,68 @@ mp_diag_h(const MainParams p) {
             dlt[u] = (int)delta[u]; lo32[u] = (int)lo[u]; hi32[u] = (int)hi[u];
         }
 
-        // seeds at each cell's first row: Mixed -> FP32 operands and compensated FP32
-        // accumulation rounded to half (FP32 precalc); FP16 -> half arithmetic throughout
-        // seeds (at the pair's first rows, then every H rows at warp-uniform steps):
-        // Mixed -> FP32 operands and FP32 accumulation rounded to half (the FP32 precalc);
-        // FP16 -> half arithmetic.  The row window is shared by the pair and the second cell's
-        // column window is the first one shifted by one position.
+        // seeds (at the pair's first rows, then every H rows at warp-uniform steps): direct
+        // centred dot products (reading G8).  Mixed -> FP32 operands and
+        // accumulation rounded to half (the FP32 precalc); FP16 -> half arithmetic; FP16C ->
+        // half arithmetic with Kahan compensation.  When both cells start on the same row the
+        // row window is shared and the second column window is the first shifted by one.
         __half2 QT[DL];
         auto seed_pair = [&](bool ok0, bool ok1, long long row0, long long row1) {
-            using TA = typename std::conditional<MIXED, float, __half>::type;
+            using TA = TS;
             const bool same = ok0 && ok1 && row0 == row1;
-            TA acc0[DL], acc1[DL];
+            TA acc0[DL], acc1[DL], cp0[DL], cp1[DL];
 #pragma unroll
-            for (int kk = 0; kk < DL; ++kk) { acc0[kk] = (TA)0.f; acc1[kk] = (TA)0.f; }
-#pragma unroll 1
-            for (int u = 0; u < (same ? 1 : 2); ++u) {
-                const bool ok = u == 0 ? ok0 : ok1;
-                if (!ok) continue;
-                const long long i0 = u == 0 ? row0 : row1, j0 = i0 + delta[u];
-                TA mq[DL], mr0[DL], mr1[DL];
-#pragma unroll
-                for (int kk = 0; kk < DL; ++kk) {
-                    mq[kk] = mu_q[i0 * D + kk * G + g];
-                    mr0[kk] = mu_r[j0 * D + kk * G + g];
-                    mr1[kk] = same ? mu_r[(j0 + 1) * D + kk * G + g] : mr0[kk];
+            for (int kk = 0; kk < DL; ++kk) { acc0[kk] = (TA)0.f; acc1[kk] = (TA)0.f; cp0[kk] = (TA)0.f; cp1[kk] = (TA)0.f; }
+            auto kadd = [](TA& acc, TA& cp, TA v) {
+                if constexpr (MODE == 2) {  // compensated half accumulation
+                    const TA y = v - cp;
+                    const TA t2 = acc + y;
+                    cp = (t2 - acc) - y;
+                    acc = t2;
+                } else {
+                    acc = acc + v;
                 }
-                TA xr_prev[DL], cp0[DL], cp1[DL];  // Kahan compensators (FP16C)
-#pragma unroll
-                for (int kk = 0; kk < DL; ++kk) { xr_prev[kk] = tw_r[j0 * D + kk * G + g]; cp0[kk] = (TA)0.f; cp1[kk] = (TA)0.f; }
+            };
+            if (same) {
+                const long long i0 = row0, j0 = row0 + delta[0];
+                TA mq[DL], mr0[DL], mr1[DL], xr[DL];
+                ldv<TA, DL, G>(mu_q + i0 * D, g, mq);
+                ldv<TA, DL, G>(mu_r + j0 * D, g, mr0);
+                ldv<TA, DL, G>(mu_r + (j0 + 1) * D, g, mr1);
+                ldv<TA, DL, G>(tw_r + j0 * D, g, xr);
 #pragma unroll 2
                 for (int tt = 0; tt < m; ++tt) {
+                    TA xq[DL], xn[DL];
+                    ldv<TA, DL, G>(tw_q + (i0 + tt) * D, g, xq);
+                    ldv<TA, DL, G>(tw_r + (j0 + tt + 1) * D, g, xn);   // j0 + m <= L - 1 (cell 1 valid)
 #pragma unroll
                     for (int kk = 0; kk < DL; ++kk) {
-                        const TA xq = tw_q[(i0 + tt) * D + kk * G + g];
-                        const TA xr = xr_prev[kk];
-                        const TA xn = tw_r[(j0 + tt + 1) * D + kk * G + g];
-                        if constexpr (MODE == 2) {  // compensated half accumulation
-                            auto kadd = [](TA& acc, TA& cp, TA v) {
-                                const TA y = v - cp;
-                                const TA t2 = acc + y;
-                                cp = (t2 - acc) - y;
-                                acc = t2;
-                            };
-                            if (same) {
-                                kadd(acc0[kk], cp0[kk], (xq - mq[kk]) * (xr - mr0[kk]));
-                                kadd(acc1[kk], cp1[kk], (xq - mq[kk]) * (xn - mr1[kk]));
-                            } else {
-                                kadd(u == 0 ? acc0[kk] : acc1[kk], u == 0 ? cp0[kk] : cp1[kk], (xq - mq[kk]) * (xr - mr0[kk]));
-                            }
-                        } else if (same) {
-                            acc0[kk] = acc0[kk] + (xq - mq[kk]) * (xr - mr0[kk]);
-                            acc1[kk] = acc1[kk] + (xq - mq[kk]) * (xn - mr1[kk]);
-                        } else {
-                            TA& acc = u == 0 ? acc0[kk] : acc1[kk];
-                            acc = acc + (xq - mq[kk]) * (xr - mr0[kk]);
-                        }
-                        xr_prev[kk] = xn;
+                        const TA cq = xq[kk] - mq[kk];
+                        kadd(acc0[kk], cp0[kk], cq * (xr[kk] - mr0[kk]));
+                        kadd(acc1[kk], cp1[kk], cq * (xn[kk] - mr1[kk]));
+                        xr[kk] = xn[kk];
                     }
+                }
+            } else {
+#pragma unroll 1
+                for (int u = 0; u < 2; ++u) {
+                    if (!(u == 0 ? ok0 : ok1)) continue;
+                    const long long i0 = u == 0 ? row0 : row1, j0 = i0 + delta[u];
+                    TA mq[DL], mr[DL], acc[DL], cp[DL];
+                    ldv<TA, DL, G>(mu_q + i0 * D, g, mq);
+                    ldv<TA, DL, G>(mu_r + j0 * D, g, mr);
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) { acc[kk] = (TA)0.f; cp[kk] = (TA)0.f; }
+#pragma unroll 2
+                    for (int tt = 0; tt < m; ++tt) {
+                        TA xq[DL], xr[DL];
+                        ldv<TA, DL, G>(tw_q + (i0 + tt) * D, g, xq);
+                        ldv<TA, DL, G>(tw_r + (j0 + tt) * D, g, xr);
+#pragma unroll
+                        for (int kk = 0; kk < DL; ++kk) kadd(acc[kk], cp[kk], (xq[kk] - mq[kk]) * (xr[kk] - mr[kk]));
+                    }
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) { if (u == 0) acc0[kk] = acc[kk]; else acc1[kk] = acc[kk]; }
                 }
             }
 #pragma unroll
@@ -279,16 +285,15 @@ mp_diag_h(const MainParams p) {
         const int s_end = nrows + CW * (RA - 1);
         const int R0 = (int)r0, C0 = (int)(r0 + delta0);
         int row_in = min(SB, nrows), col_in = min(SB, s_end) + CW;  // pairs need column c+1's slot too
-        int row_out = 0, col_out = 0;
-        int fx_r0 = 0, fx_r1 = row_in, fx_c0 = 0, fx_c1 = col_in;
+        int fx_r0 = 0, fx_c0 = 0;
         stage(true, R0, 0, row_in);
         stage(false, C0, 0, col_in);
         cp_async_commit();
         cp_async_wait_all();
         __syncwarp();
-        fixup(true, R0, fx_r0, fx_r1);
-        fixup(false, C0, fx_c0, fx_c1);
-        fx_r0 = fx_r1; fx_c0 = fx_c1;
+        fixup(true, R0, 0, row_in);
+        fixup(false, C0, 0, col_in);
+        fx_r0 = row_in; fx_c0 = col_in;
         __syncwarp();
 
         auto step = [&](int s) {
@@ -303,29 +308,29 @@ mp_diag_h(const MainParams p) {
                 upd[u] = row > lo32[u] && row < hi32[u];
             }
             if (s == seeded_step) upd[0] = upd[1] = false;  // QT of this row was just seeded
-            __half2 S[DL], tr[DL], tc[DL];
+            // D (Eq. 1) for both cells; threshold = max of the row's and the column's best
+            // (a cell can improve either iff S_k <= that max)
+            __half2 S[DL], th[DL];
             if (upd[0] == upd[1]) {
 #pragma unroll
                 for (int kk = 0; kk < DL; ++kk) {
                     const int pl = kk * G + g;
-                    const H4 R = rowv[pl * PSR + sr];
+                    const RH R = rowv[pl * PSR + sr];
                     const H4 C = colv[pl * PSC + scn];
-                    if (upd[0]) QT[kk] = __hfma2(R.x, C.y, __hfma2(C.x, R.y, QT[kk]));   // Eq. (1)
-                    S[kk] = h2sqrt(__habs2(__hfma2(__hneg2(QT[kk]), __hmul2(R.z, C.z), two_m)));
-                    tr[kk] = R.w;
-                    tc[kk] = C.w;
+                    if (upd[0]) QT[kk] = __hfma2(__half2half2(R.df), C.y, __hfma2(C.x, __half2half2(R.dg), QT[kk]));
+                    S[kk] = h2sqrt(__habs2(__hfma2(__hneg2(QT[kk]), __hmul2(__half2half2(R.a), C.z), two_m)));
+                    th[kk] = SELF ? __hmax2(__half2half2(R.t), C.w) : __half2half2(R.t);
                 }
             } else {  // the two cells of the pair are at different phases (tile / diagonal start)
                 const __half2 msk = __halves2half2(__float2half(upd[0] ? 1.f : 0.f), __float2half(upd[1] ? 1.f : 0.f));
 #pragma unroll
                 for (int kk = 0; kk < DL; ++kk) {
                     const int pl = kk * G + g;
-                    const H4 R = rowv[pl * PSR + sr];
+                    const RH R = rowv[pl * PSR + sr];
                     const H4 C = colv[pl * PSC + scn];
-                    QT[kk] = __hfma2(msk, __hfma2(R.x, C.y, __hmul2(C.x, R.y)), QT[kk]);
-                    S[kk] = h2sqrt(__habs2(__hfma2(__hneg2(QT[kk]), __hmul2(R.z, C.z), two_m)));
-                    tr[kk] = R.w;
-                    tc[kk] = C.w;
+                    QT[kk] = __hfma2(msk, __hfma2(__half2half2(R.df), C.y, __hmul2(C.x, __half2half2(R.dg))), QT[kk]);
+                    S[kk] = h2sqrt(__habs2(__hfma2(__hneg2(QT[kk]), __hmul2(__half2half2(R.a), C.z), two_m)));
+                    th[kk] = SELF ? __hmax2(__half2half2(R.t), C.w) : __half2half2(R.t);
                 }
             }
             sort_net<__half2, DL>(S);                                              // Eq. (2)
@@ -346,13 +351,13 @@ mp_diag_h(const MainParams p) {
             }
             unsigned hm[4] = {0u, 0u, 0u, 0u};
 #pragma unroll
-            for (int kk = 0; kk < DL; ++kk) {
-                hm[kk & 3] |= __hle2_mask(S[kk], tr[kk]);
-                if (SELF) hm[kk & 3] |= __hle2_mask(S[kk], tc[kk]);
-            }
+            for (int kk = 0; kk < DL; ++kk) hm[kk & 3] |= __hle2_mask(S[kk], th[kk]);
             const unsigned hmask = (hm[0] | hm[1]) | (hm[2] | hm[3]);
             const bool hit = ((hmask & 0xffffu) && active[0]) || ((hmask >> 16) && active[1]);
             if (__any_sync(FULL, hit)) {
+                // Eq. (3): group min by shuffles; the leader of a row / column group compares
+                // with the ring's best and writes an improvement (or a tie, for the index
+                // rule) through to the merge key.
 #pragma unroll
                 for (int kk = 0; kk < DL; ++kk) {
                     __half2 v = S[kk];
@@ -364,29 +369,29 @@ mp_diag_h(const MainParams p) {
 #pragma unroll 1
                 for (int kk = 0; kk < DL; ++kk) {
                     const int pl = kk * G + g;
+                    const int rk = g * DL + kk;  // rank held in register kk after the merge
                     const __half2 vh = ssc[kk * 32 + lane];
                     const float v[2] = {__low2float(vh), __high2float(vh)};
-                    const bool need_r = __any_sync(FULL, fminf(v[0], v[1]) <= rowb[pl * PSR + sr]);
-                    bool need_c = false;
-                    if (SELF) need_c = __any_sync(FULL, v[0] <= colb[pl * PSC + scn] ||
-                                                      v[1] <= colb[pl * PSC + Gm::scol(col0 + 1)]);
-                    if (!need_r && !need_c) continue;
-                    float vr = fminf(v[0], v[1]);
+                    const int ixr = pl * PSR + sr;
+                    const float tr = __half2float(rowv[ixr].t);
+                    float tc[2] = {-FINF, -FINF};
+                    if (SELF) {
+                        const __half2 w = colv[pl * PSC + scn].w;
+                        tc[0] = __low2float(w);
+                        tc[1] = __high2float(w);
+                    }
+                    const bool need_r = __any_sync(FULL, fminf(v[0], v[1]) <= tr);
+                    const bool need_c = SELF && __any_sync(FULL, v[0] <= tc[0] || v[1] <= tc[1]);
+                    if (need_r) {
+                        float vr = fminf(v[0], v[1]);
 #pragma unroll
-                    for (int bit = 0; bit < Gm::LOG_CA; ++bit)
-                        vr = fminf(vr, __shfl_xor_sync(FULL, vr, 1 << (bit + Gm::LOG_G)));
-                    const bool mine = v[0] == vr || v[1] == vr;
-                    const unsigned eqr = __ballot_sync(FULL, mine) & gmask_row;
-                    if (need_r && vr < FINF && lane == __ffs(eqr) - 1) {
-                        const int j = (v[0] == vr) ? col0 : col0 + 1;          // lowest column first
-                        const int ix = pl * PSR + sr;
-                        const float cur = rowb[ix];
-                        const unsigned ci = rowi[ix] & ~DIRTY;
-                        if (vr < cur || (vr == cur && (unsigned)j < ci)) {
-                            rowb[ix] = vr;
-                            rowi[ix] = (unsigned)j | DIRTY;
-                            rowv[ix].w = __float2half2_rn(vr);
-                            rowdirty[sr] = 1;
+                        for (int bit = 0; bit < Gm::LOG_CA; ++bit)
+                            vr = fminf(vr, __shfl_xor_sync(FULL, vr, 1 << (bit + Gm::LOG_G)));
+                        const unsigned eqr = __ballot_sync(FULL, v[0] == vr || v[1] == vr) & gmask_row;
+                        if (vr < FINF && vr <= tr && lane == __ffs(eqr) - 1) {
+                            const int j = (v[0] == vr) ? col0 : col0 + 1;          // lowest column first
+                            KeyOps<float>::merge(keys + (size_t)row * d + rk, vr, (unsigned)j);
+                            if (vr < tr) rowv[ixr].t = __float2half_rn(vr);        // exact
                         }
                     }
                     if (SELF && need_c) {
@@ -397,19 +402,14 @@ mp_diag_h(const MainParams p) {
                             for (int bit = 0; bit < 5 - Gm::LOG_G - Gm::LOG_CA; ++bit)
                                 vc = fminf(vc, __shfl_xor_sync(FULL, vc, 1 << (bit + Gm::LOG_G + Gm::LOG_CA)));
                             const unsigned eqc = __ballot_sync(FULL, v[u] == vc) & gmask_col;
-                            if (vc < FINF && eqc != 0 && lane == 31 - __clz(eqc)) {
+                            // lowest row index = highest a = highest lane
+                            if (vc < FINF && vc <= tc[u] && eqc != 0 && lane == 31 - __clz(eqc)) {
                                 const int colu = col0 + u;
-                                const int scu = Gm::scol(colu);
-                                const int ix = pl * PSC + scu;
-                                const float cur = colb[ix];
-                                const unsigned ci = coli[ix] & ~DIRTY;
-                                if (vc < cur || (vc == cur && (unsigned)row < ci)) {
-                                    colb[ix] = vc;
-                                    coli[ix] = (unsigned)row | DIRTY;
+                                KeyOps<float>::merge(keys + (size_t)colu * d + rk, vc, (unsigned)row);
+                                if (vc < tc[u]) {
                                     const __half h = __float2half_rn(vc);
-                                    reinterpret_cast<__half*>(&colv[ix].w)[0] = h;
+                                    reinterpret_cast<__half*>(&colv[pl * PSC + Gm::scol(colu)].w)[0] = h;
                                     reinterpret_cast<__half*>(&colv[pl * PSC + Gm::scol(colu - 1)].w)[1] = h;
-                                    coldirty[scu] = 1;
                                 }
                             }
                         }
@@ -430,17 +430,13 @@ mp_diag_h(const MainParams p) {
                 }
                 seeded_step = s0 == 0 ? -1 : s0;
             }
-            const int rx = min(max(s0 - CW * (RA - 1), 0), nrows);
-            evict(true, R0, row_out, rx);
-            row_out = rx;
-            evict(false, C0, col_out, s0);
-            col_out = s0;
+            // prefetch the next batch's entries (positions older than this batch are dead:
+            // the rings hold exactly the live span, bests were written through)
             const int nxt = min(s0 + 2 * SB, s_end);
             const int r_need = min(nxt, nrows), c_need = nxt + CW;
             stage(true, R0, row_in, r_need);
             stage(false, C0, col_in, c_need);
-            fx_r1 = max(row_in, r_need);
-            fx_c1 = max(col_in, c_need);
+            const int fx_r1 = max(row_in, r_need), fx_c1 = max(col_in, c_need);
             row_in = fx_r1;
             col_in = fx_c1;
             cp_async_commit();
@@ -455,8 +451,6 @@ mp_diag_h(const MainParams p) {
             fx_c0 = fx_c1;
             __syncwarp();
         }
-        evict(true, R0, row_out, nrows);
-        evict(false, C0, col_out, col_in);
         __syncwarp();
     }
 }

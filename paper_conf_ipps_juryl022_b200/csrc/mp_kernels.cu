@@ -228,11 +228,10 @@ __global__ void pre_fmt_h(const PreParams p) {
     q.z = __halves2half2(va ? f[2 * nd + ia] : z, vb ? f[2 * nd + ib] : z);
     q.w = __half2half2(z);
     reinterpret_cast<H4*>(p.st_pair)[gid] = q;
-    if (vb) {
-        H4 r;
-        r.x = __half2half2(f[ib]); r.y = __half2half2(f[nd + ib]); r.z = __half2half2(f[2 * nd + ib]);
-        r.w = __half2half2(z);
-        reinterpret_cast<H4*>(p.st)[ib] = r;
+    if (vb) {  // row format: one position (the kernel broadcasts it to both cells of a pair)
+        RH r;
+        r.df = f[ib]; r.dg = f[nd + ib]; r.a = f[2 * nd + ib]; r.t = z;
+        reinterpret_cast<RH*>(p.st)[ib] = r;
     }
 }
 template <class T>
@@ -320,7 +319,7 @@ Variant pick_variant(int prec, int d) {
     while (dp < d) dp <<= 1;
     Variant v;
     if (prec == P16 || prec == PMIX || prec == P16C) {  // half2: a lane-cell is a pair of diagonals
-        if (dp <= 8) { v.DL = dp; v.G = 1; }
+        if (dp <= 16) { v.DL = dp; v.G = 1; }
         else if (dp <= 256) { v.DL = 8; v.G = dp / 8; }
         else { v.DL = dp / 32; v.G = 32; }
         v.W = 2;
@@ -364,7 +363,7 @@ static long long dispatch_h(int op, int DL, int G, const MainParams* p, int grid
         if (op == 3) return InstH<dl, g, SELF, MIXED>::warps_per_block();                  \
         return InstH<dl, g, SELF, MIXED>::blocks_per_sm();                                 \
     }
-    MP_HCASE(1, 1) MP_HCASE(2, 1) MP_HCASE(4, 1) MP_HCASE(8, 1)
+    MP_HCASE(1, 1) MP_HCASE(2, 1) MP_HCASE(4, 1) MP_HCASE(8, 1) MP_HCASE(16, 1)
     MP_HCASE(8, 2) MP_HCASE(8, 4) MP_HCASE(8, 8) MP_HCASE(8, 16) MP_HCASE(8, 32) MP_HCASE(16, 32) MP_HCASE(32, 32)
 #undef MP_HCASE
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
