@@ -45,6 +45,20 @@
 #ifndef MP_KEEP_DL
 #define MP_KEEP_DL 16
 #endif
+#ifndef MP_SEED_CHUNK
+#define MP_SEED_CHUNK 4
+#endif
+// steps per staging batch by lanes-per-cell G: wide cells (large d) keep fewer positions in
+// flight so the per-warp rings stay small enough for several resident warps per SM
+#ifndef MP_SB_G1
+#define MP_SB_G1 4
+#endif
+#ifndef MP_SB_G2
+#define MP_SB_G2 2
+#endif
+#ifndef MP_SB_G4
+#define MP_SB_G4 1
+#endif
 
 namespace mpk {
 
@@ -256,7 +270,7 @@ template <int G, int W> struct Geo {
     static constexpr int NC = NL * W;                                    // cells (diagonals) per warp
     // ring positions move in batches of SB steps, prefetched one batch ahead: live rows
     // span CW(RA-1) + 2 SB, live columns 2 SB + CW - 1
-    static constexpr int SB = 4;
+    static constexpr int SB = G == 1 ? MP_SB_G1 : G == 2 ? MP_SB_G2 : MP_SB_G4;
     static constexpr int RING_R = pow2ceil(CW * (RA - 1) + 2 * SB) < CW ? CW : pow2ceil(CW * (RA - 1) + 2 * SB);
     static constexpr int RPC = RING_R / CW;                              // ring rows per residue class
     static constexpr int RING_C = pow2ceil(2 * SB + CW - 1);
@@ -469,30 +483,36 @@ mp_diag(const MainParams p) {
         // position-major and padded to D dims, so a lane (G == 1) loads its DL dims as vectors.
         T QT[W][DL];
         auto seed_cell = [&](int u, long long row) {
-            T mq[DL], mr[DL], cmp[DL];
+            // dims in chunks of SC: the m-long dot-product loop then keeps few operand
+            // registers live, so seeding never sets the kernel's register peak
+            constexpr int SC = (DL % MP_SEED_CHUNK == 0) ? MP_SEED_CHUNK : DL;
             const long long i0 = row, j0 = row + delta[u];
-            load_dims<T, DL, G>(mu_q + i0 * D, g, mq);
-            load_dims<T, DL, G>(mu_r + j0 * D, g, mr);
-#pragma unroll
-            for (int kk = 0; kk < DL; ++kk) { QT[u][kk] = (T)0; cmp[kk] = (T)0; }
             const T* xq_p = tw_q + i0 * D;
             const T* xr_p = tw_r + j0 * D;
+#pragma unroll
+            for (int c0 = 0; c0 < DL; c0 += SC) {
+                T mq[SC], mr[SC], cmp[SC], acc[SC];
+                load_dims<T, SC, G>(mu_q + i0 * D + c0 * G, g, mq);
+                load_dims<T, SC, G>(mu_r + j0 * D + c0 * G, g, mr);
+#pragma unroll
+                for (int kk = 0; kk < SC; ++kk) { acc[kk] = (T)0; cmp[kk] = (T)0; }
 #pragma unroll 2
-            for (int tt = 0; tt < m; ++tt) {
-                T xq[DL], xr[DL];
-                load_dims<T, DL, G>(xq_p + (long long)tt * D, g, xq);
-                load_dims<T, DL, G>(xr_p + (long long)tt * D, g, xr);
+                for (int tt = 0; tt < m; ++tt) {
+                    T xq[SC], xr[SC];
+                    load_dims<T, SC, G>(xq_p + (long long)tt * D + c0 * G, g, xq);
+                    load_dims<T, SC, G>(xr_p + (long long)tt * D + c0 * G, g, xr);
 #pragma unroll
-                for (int kk = 0; kk < DL; ++kk) {
-                    const T y = (xq[kk] - mq[kk]) * (xr[kk] - mr[kk]) - cmp[kk];
-                    const T t2 = QT[u][kk] + y;
-                    cmp[kk] = (t2 - QT[u][kk]) - y;
-                    QT[u][kk] = t2;
+                    for (int kk = 0; kk < SC; ++kk) {
+                        const T y = (xq[kk] - mq[kk]) * (xr[kk] - mr[kk]) - cmp[kk];
+                        const T t2 = acc[kk] + y;
+                        cmp[kk] = (t2 - acc[kk]) - y;
+                        acc[kk] = t2;
+                    }
                 }
-            }
 #pragma unroll
-            for (int kk = 0; kk < DL; ++kk)
-                if ((kk * G + g) >= d) QT[u][kk] = (T)-1;  // padded dims (zero data)
+                for (int kk = 0; kk < SC; ++kk)
+                    QT[u][c0 + kk] = ((c0 + kk) * G + g) >= d ? (T)-1 : acc[kk];  // padded dims: zero data
+            }
         };
 #pragma unroll
         for (int u = 0; u < W; ++u) {
@@ -694,10 +714,12 @@ mp_diag(const MainParams p) {
             }
         };
 
+        int to_seed = H;  // steps until the next re-seed (H is a multiple of SB)
         for (int s0 = 0; s0 < s_end; s0 += SB) {
             // seeds: each cell's first row at s0 = 0, then the current row every H steps
             // (H is a multiple of SB, so re-seeds fall on batch starts: one call site)
-            if (s0 > 0 && s0 % H == 0) {
+            if (s0 > 0 && (to_seed -= SB) == 0) {
+                to_seed = H;
                 const long long row = R0 + s0 - (long long)CW * a;
 #pragma unroll 1
                 for (int u = 0; u < W; ++u)

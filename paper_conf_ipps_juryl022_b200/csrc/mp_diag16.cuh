@@ -419,8 +419,10 @@ mp_diag_h(const MainParams p) {
             }
         };
 
+        int to_seed = SB;  // steps until the next seed (H is a multiple of SB)
         for (int s0 = 0; s0 < s_end; s0 += SB) {
-            if (s0 % H == 0) {  // seeds: first rows at s0 = 0, current row every H steps
+            if ((to_seed -= SB) == 0) {  // seeds: first rows at s0 = 0, current row every H steps
+                to_seed = H;
                 const long long row = R0 + s0 - (long long)CW * a;
                 if (s0 == 0) {
                     seed_pair(lo[0] < hi[0], lo[1] < hi[1], lo[0], lo[1]);

@@ -346,8 +346,10 @@ mp_diag64f(const MainParams p) {
             __syncwarp();
         };
 
+        int to_seed = SB;  // steps until the next seed (H is a multiple of SB)
         for (int s0 = 0; s0 < s_end; s0 += SB) {
-            if (s0 % H == 0) {  // seeds: first row at s0 = 0, current row every H steps
+            if ((to_seed -= SB) == 0) {  // seeds: first row at s0 = 0, current row every H steps
+                to_seed = H;
                 const long long row = R0 + s0 - (long long)CW * a;
                 if (s0 == 0) { if (lo < hi) seed_cell(lo); }
                 else if (row > lo && row < hi) seed_cell(row);
