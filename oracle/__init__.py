@@ -41,7 +41,9 @@ def _load():
         lib.oracle_cell.argtypes = [p, p, i64, i64, i64, i64, i64, p]
         lib.oracle_mstamp.argtypes = [p, p, i64, i64, i64, i64, p, i64, ctypes.c_int, p, p, p]
         lib.oracle_cells.argtypes = [p, p, i64, i64, i64, p, p, i64, p]
-        for f in (lib.oracle_window_stats, lib.oracle_cell, lib.oracle_mstamp, lib.oracle_cells):
+        lib.oracle_mstamp_band.argtypes = [p, p, i64, i64, i64, i64, p, i64, i64, i64, ctypes.c_int, p, p, p]
+        for f in (lib.oracle_window_stats, lib.oracle_cell, lib.oracle_mstamp, lib.oracle_cells,
+                  lib.oracle_mstamp_band):
             f.restype = ctypes.c_int
         _lib = lib
     return _lib
@@ -125,5 +127,27 @@ def mstamp(T, m, exclusion=None, Tr=None, rows=None, nthreads=None):
     nt = nthreads or os.cpu_count() or 1
     rc = _load().oracle_mstamp(_ptr(T), _ptr(Tr_), d, n, m, int(exclusion), _ptr(r), nrows,
                                int(nt), _ptr(P), _ptr(I), _ptr(P2))
+    assert rc == 0
+    return P, I, P2
+
+
+def mstamp_band(T, m, rows, dlo, dhi, exclusion=None, Tr=None, nthreads=None):
+    """Partial profile of one diagonal band for query rows: min / argmin /
+    runner-up over the cells with delta = j - i (AB-join) or |j - i| (self-join) in
+    [dlo, dhi), self-join exclusion as in mstamp().  Returns (P, I, P2), each (d, len(rows))."""
+    T = _series(T)
+    d, L = T.shape
+    n = L - m + 1
+    if exclusion is None or exclusion < 0:
+        exclusion = -(-m // 4)
+    Tr_ = None if Tr is None else _series(Tr)
+    r = np.ascontiguousarray(rows, dtype=np.int64)
+    nrows = len(r)
+    P = np.empty((d, nrows))
+    P2 = np.empty((d, nrows))
+    I = np.empty((d, nrows), dtype=np.int64)
+    nt = nthreads or os.cpu_count() or 1
+    rc = _load().oracle_mstamp_band(_ptr(T), _ptr(Tr_), d, n, m, int(exclusion), _ptr(r), nrows,
+                                    int(dlo), int(dhi), int(nt), _ptr(P), _ptr(I), _ptr(P2))
     assert rc == 0
     return P, I, P2

@@ -283,3 +283,58 @@ def test_c3_sampled_rows(ctx, oracle_mod, prec):
     for k in range(32):
         assert abs(Ig[k, a] - b) <= slack and abs(Ig[k, b] - a) <= slack
     assert np.all(np.diff(Pg, axis=0) >= -1e-3 * Pg[1:])
+
+
+# ---------------------------------------------------------------- C4 / C5 at full size, one band
+@pytest.mark.parametrize("cfg_name,prec,world", [("C4", "fp32", 512), ("C4", "fp64", 1024),
+                                                 ("C5", "fp32", 1024), ("C5", "mixed", 1024)])
+def test_full_size_band_sampled_rows(ctx, oracle_mod, cfg_name, prec, world):
+    """BASELINE configs C4 (AB-join d=128, n=2^20, m=256) and C5 (self-join d=256, n=2^21,
+    m=512) at full input size: one diagonal band of a world-way split (the per-GPU unit of
+    SURVEY 8(e), computed by mp_partial_device exactly as one rank of bench.py --gpus N does)
+    is finalized and its sampled rows checked against the oracle's partial profile of the
+    same band (oracle.mstamp_band).  The band is the one holding the planted motif's
+    diagonal, so the motif must be recovered at full size."""
+    from paper_conf_ipps_juryl022_b200 import mstamp
+    cfg = datagen.make(cfg_name)
+    T, Tr, m, e, n, d = cfg["T"], cfg["Tr"], cfg["m"], cfg["exclusion"], cfg["n"], cfg["d"]
+    self_join = Tr is None
+    a, b = datagen.motif_positions(n, m)
+    db = mstamp.plan_diagonals(d, n, m, prec, e, self_join, world)
+    rank = int(np.searchsorted(db, b - a, side="right") - 1)
+    dlo, dhi = int(db[rank]), int(db[rank + 1])
+    assert dlo <= b - a < dhi
+    Td = torch.from_numpy(T).cuda()
+    Trd = None if self_join else torch.from_numpy(Tr).cuda()
+    keys = torch.empty(mstamp.key_words(d, n, prec), dtype=torch.int64, device="cuda")
+    ctx.partial_device(Td, m, keys, rank, world, prec, e, Tr=Trd)
+    Pd = torch.empty(d, n, dtype=torch.float64, device="cuda")
+    Id = torch.empty(d, n, dtype=torch.int64, device="cuda")
+    ctx.finalize_device(d, n, keys, Pd, Id, prec)
+    Pg, Ig = Pd.cpu().numpy(), Id.cpu().numpy()
+    del Td, Trd, keys, Pd, Id
+    rng = np.random.default_rng(7)
+    # rows the band reaches: i + delta in [0, n) (and, self-join, i - delta >= 0)
+    hi_row = n - max(dlo, 0)
+    cand = rng.integers(0, hi_row, 6) if self_join is False else rng.integers(0, n, 6)
+    rows = np.unique(np.concatenate([[a, b, 0, n - 1], cand]))
+    P, I, P2 = oracle_mod.mstamp_band(T, m, rows, dlo, dhi, e, Tr=Tr)
+    if prec in ("fp32", "fp64"):
+        st = parity.check(oracle_mod, T, m, P, I, P2, Pg, Ig, prec, rows=rows, Tr=Tr)
+    else:
+        fin = np.isfinite(P)
+        assert np.array_equal(fin, np.isfinite(Pg[:, rows]))
+        st = _half_stats(np.where(fin, P, 1.0), I, np.where(fin, Pg[:, rows], 1.0), Ig[:, rows], m)
+        assert st["median_rel"] < 0.02
+    print(cfg_name, prec, "band", rank, "of", world, (dlo, dhi), st)
+    # planted motif (row a's partner b lies on this band's diagonal b - a)
+    slack = 0 if prec in ("fp32", "fp64") else m // 16
+    for k in range(max(1, d // 2)):
+        assert abs(Ig[k, a] - b) <= slack
+        if self_join:
+            assert abs(Ig[k, b] - a) <= slack
+    # properties at every row of the band partial: bound and monotone in k
+    fin = np.isfinite(Pg)
+    assert np.all(Pg[fin] >= 0) and np.all(Pg[fin] <= 2 * math.sqrt(m) * 1.01)
+    with np.errstate(invalid="ignore"):
+        assert np.all(np.nan_to_num(np.diff(Pg, axis=0), nan=0.0, posinf=0.0) >= -1e-3 * np.nan_to_num(Pg[1:], posinf=0.0))

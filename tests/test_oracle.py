@@ -248,3 +248,70 @@ def test_reading_g7_recurrence_identity():
             i, j = i0 + s, j0 + s
             q = q + dfx[i] * dgy[j] + dfy[j] * dgx[i]
             assert abs(q - QT[i, j]) <= 1e-9 * (1 + abs(QT[i, j]))
+
+
+# ---------------------------------------------------------------- band partials
+def _lexmin(parts):
+    """(value, index) lexicographic min over band partials (the MINLOC merge, reading G2)."""
+    P = np.full_like(parts[0][0], np.inf)
+    I = np.full_like(parts[0][1], -1)
+    for Pb, Ib in parts:
+        Ib_key = np.where(Ib < 0, np.iinfo(np.int64).max, Ib)
+        I_key = np.where(I < 0, np.iinfo(np.int64).max, I)
+        take = (Pb < P) | ((Pb == P) & (Ib_key < I_key))
+        P = np.where(take, Pb, P)
+        I = np.where(take, Ib, I)
+    return P, I
+
+
+@pytest.mark.parametrize("ab", [False, True])
+def test_band_all_diagonals_equals_rows(oracle_mod, ab):
+    """A band covering every diagonal is the sampled-row profile, bit for bit."""
+    d, n, m, e = 3, 300, 16, 4
+    if ab:
+        T, Tr = datagen.random_walk_ab(d, n, m, 61)
+        dlo, dhi = -(n - 1), n
+    else:
+        T, Tr = datagen.random_walk(d, n, m, 61), None
+        dlo, dhi = e + 1, n
+    rows = np.arange(0, n, 7)
+    P, I, P2 = oracle_mod.mstamp(T, m, e, Tr=Tr, rows=rows)
+    Pb, Ib, P2b = oracle_mod.mstamp_band(T, m, rows, dlo, dhi, e, Tr=Tr)
+    assert np.array_equal(P, Pb) and np.array_equal(I, Ib) and np.array_equal(P2, P2b)
+
+
+@pytest.mark.parametrize("ab", [False, True])
+def test_band_partition_merges_to_full(oracle_mod, ab):
+    """Disjoint bands merged by lexicographic (value, index) min give the full profile."""
+    d, n, m, e = 4, 260, 12, 3
+    if ab:
+        T, Tr = datagen.random_walk_ab(d, n, m, 62)
+        cuts = [-(n - 1), -40, 0, 1, 90, n]
+    else:
+        T, Tr = datagen.random_walk(d, n, m, 62), None
+        cuts = [e + 1, 9, 60, 61, n]
+    rows = np.arange(n)
+    P, I, _ = oracle_mod.mstamp(T, m, e, Tr=Tr)
+    parts = [oracle_mod.mstamp_band(T, m, rows, a, b, e, Tr=Tr)[:2] for a, b in zip(cuts[:-1], cuts[1:])]
+    Pm, Im = _lexmin(parts)
+    assert np.array_equal(Pm, P) and np.array_equal(Im, I)
+
+
+def test_band_vs_bruteforce(oracle_mod):
+    """One band against the definitional brute force restricted to the band's cells."""
+    d, n, m, e = 3, 90, 10, 2
+    T = datagen.random_walk(d, n, m, 63, motif=False)
+    D = brute.dist_cube(T, m)
+    dlo, dhi = 20, 45
+    rows = np.arange(n)
+    Pb, Ib, _ = oracle_mod.mstamp_band(T, m, rows, dlo, dhi, e)
+    for i in range(n):
+        best = np.full(d, np.inf)
+        for j in range(n):
+            if not (dlo <= abs(j - i) < dhi) or abs(i - j) <= e:
+                continue
+            s = np.cumsum(np.sort(D[:, i, j])) / np.arange(1, d + 1)
+            best = np.minimum(best, s)
+        fin = np.isfinite(best)
+        assert np.array_equal(fin, np.isfinite(Pb[:, i]))
+        assert np.allclose(Pb[fin, i], best[fin], rtol=1e-11, atol=1e-12)
