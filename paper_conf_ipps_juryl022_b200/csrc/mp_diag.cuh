@@ -236,6 +236,12 @@ template <> struct KeyOps<double> {
     }
 };
 
+// Warp OR of a 64-bit mask (two REDUX.OR).
+__device__ __forceinline__ unsigned long long or_reduce(unsigned long long v) {
+    const unsigned lo = __reduce_or_sync(FULL, (unsigned)v), hi = __reduce_or_sync(FULL, (unsigned)(v >> 32));
+    return ((unsigned long long)hi << 32) | lo;
+}
+
 // Load the DL dims a lane owns (dims kk*G + g) of one position-major, D-padded row.
 template <class T, int DL, int G>
 __device__ __forceinline__ void load_dims(const T* __restrict__ rowp, int g, T (&out)[DL]) {
@@ -293,7 +299,7 @@ template <class T, int DL, int G, int W> struct Smem {
     static constexpr int D = DL * G;
     static constexpr size_t ring_bytes =
         (((size_t)D * (Gm::PSR + Gm::PSC) * (sizeof(V4) + sizeof(unsigned))) + 15) & ~(size_t)15;
-    static constexpr size_t flag_bytes = ((Gm::RING_R + Gm::RING_C) * 4 + 15) & ~(size_t)15;
+    static constexpr size_t flag_bytes = 0;  // dirty flags live in registers (bit masks)
     static constexpr size_t bytes_per_warp = ring_bytes + flag_bytes + (size_t)W * DL * 32 * sizeof(T);
     // warps per block: up to 4, fewer when a warp's rings are large (blocks <= ~112 KB)
     static constexpr int WPB = bytes_per_warp * 4 <= 112 * 1024 ? 4 : bytes_per_warp * 2 <= 112 * 1024 ? 2 : 1;
@@ -328,8 +334,11 @@ mp_diag(const MainParams p) {
     V4* colv = rowv + (size_t)D * PSR;
     unsigned* rowi = reinterpret_cast<unsigned*>(colv + (size_t)D * PSC);
     unsigned* coli = rowi + (size_t)D * PSR;
-    unsigned* rowdirty = reinterpret_cast<unsigned*>(wbase + SM::ring_bytes);
-    unsigned* coldirty = rowdirty + Gm::RING_R;
+    // dirty ring slots: warp-uniform bit masks in registers (slot -> bit), set after each
+    // slow path by a warp OR-reduction, cleared on eviction -- no shared-memory flags to poll
+    static_assert(Gm::RING_R <= 64 && Gm::RING_C <= 64, "dirty masks hold one bit per ring slot");
+    using DMask = unsigned long long;
+    DMask dmask_r = 0, dmask_c = 0;
     T* ssc = reinterpret_cast<T*>(wbase + SM::ring_bytes + SM::flag_bytes);
 
     const V4* __restrict__ st_q = reinterpret_cast<const V4*>(p.st_q);
@@ -365,7 +374,6 @@ mp_diag(const MainParams p) {
         if (cnt <= 0) return;
         V4* buf = is_row ? rowv : colv;
         unsigned* ib = is_row ? rowi : coli;
-        unsigned* dflag = is_row ? rowdirty : coldirty;
         const int ps = is_row ? PSR : PSC;
         const V4* __restrict__ st = is_row ? st_q : st_r;
         const bool want_thr = is_row || SELF;
@@ -375,7 +383,6 @@ mp_diag(const MainParams p) {
                 const int pi = e / D, pl = e - pi * D;
                 const int pos = base + p_lo + pi;
                 const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
-                if (pl == 0) dflag[sl] = 0;
                 V4* dst = &buf[pl * ps + sl];
                 const V4* src = st + (size_t)pos * d + pl;
                 if constexpr (sizeof(T) == 4) {
@@ -394,7 +401,6 @@ mp_diag(const MainParams p) {
             const int pos = base + p_lo + pi;
             if (pos < 0 || pos >= n32) continue;
             const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
-            if (pl == 0) dflag[sl] = 0;
             V4* dst = &buf[pl * ps + sl];
             const V4* src = st + (size_t)pos * d + pl;
             if (pl < d) {
@@ -423,21 +429,24 @@ mp_diag(const MainParams p) {
         if (cnt <= 0) return;
         const V4* buf = is_row ? rowv : colv;
         const unsigned* ib = is_row ? rowi : coli;
-        const unsigned* dflag = is_row ? rowdirty : coldirty;
         const int ps = is_row ? PSR : PSC;
-        // early out: most evictions find nothing dirty
-        bool any = false;
-        for (int pi = lane; pi < cnt; pi += 32) {  // one pass in steady state (cnt = SB)
+        // early out (warp-uniform, registers only): most evictions find nothing dirty
+        DMask& dm = is_row ? dmask_r : dmask_c;
+        if (dm == 0) return;
+        DMask leaving = 0;
+        for (int pi = 0; pi < cnt; ++pi) {
             const int pos = base + p_lo + pi;
-            if (pos >= 0 && pos < n32) any |= dflag[is_row ? Gm::srow(pos) : Gm::scol(pos)] != 0;
+            leaving |= 1ull << (is_row ? Gm::srow(pos) : Gm::scol(pos));
         }
-        if (!__any_sync(FULL, any)) return;
+        const DMask dirty = dm & leaving;
+        if (dirty == 0) return;
+        dm &= ~leaving;
         for (int e = lane; e < cnt * D; e += 32) {
             const int pi = e / D, pl = e - pi * D;
             const int pos = base + p_lo + pi;
             if (pos < 0 || pos >= n32) continue;
             const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
-            if (dflag[sl] == 0) continue;
+            if (((dirty >> sl) & 1ull) == 0) continue;
             const int rk = rank_of_plane<DL, G>(pl);
             if (rk >= d) continue;
             const unsigned ix = ib[pl * ps + sl];
@@ -524,6 +533,8 @@ mp_diag(const MainParams p) {
             }
         }
         int seeded_step = -1;  // step whose row was re-seeded at its batch start
+        dmask_r = 0;
+        dmask_c = 0;
 
         const int nrows = (int)(r1 - r0);
         const int s_end = nrows + CW * (RA - 1);
@@ -644,6 +655,7 @@ mp_diag(const MainParams p) {
 #pragma unroll
                     for (int kk = 0; kk < DL; ++kk) ssc[(u * DL + kk) * 32 + lane] = active[u] ? S[u][kk] : INF;
                 __syncwarp();
+                DMask mark_r = 0, mark_c = 0;  // ring slots this lane's leader updates dirtied
 #pragma unroll 1
                 for (int kk = 0; kk < DL; ++kk) {
                     const int pl = kk * G + g;
@@ -684,7 +696,7 @@ mp_diag(const MainParams p) {
                         if (vr < cur || (vr == cur && (unsigned)j < ci)) {
                             rowv[ix].w = vr;
                             rowi[ix] = (unsigned)j | DIRTY;
-                            rowdirty[sr] = 1;
+                            mark_r |= 1ull << sr;
                         }
                     }
                     if (SELF && need_c) {
@@ -704,12 +716,14 @@ mp_diag(const MainParams p) {
                                 if (vc < cur || (vc == cur && (unsigned)row < ci)) {
                                     colv[ix].w = vc;
                                     coli[ix] = (unsigned)row | DIRTY;
-                                    coldirty[scu] = 1;
+                                    mark_c |= 1ull << scu;
                                 }
                             }
                         }
                     }
                 }
+                dmask_r |= or_reduce(mark_r);
+                dmask_c |= or_reduce(mark_c);
                 __syncwarp();
             }
         };
