@@ -12,22 +12,25 @@
 // the unfiltered kernel.  Results are identical to a pure FP64 evaluation of the same cells.
 //
 // Structure as mp_diag (mp_diag.cuh): warp tiles, staggered lane-cells, cp.async-staged
-// per-warp rings (entries: df, dg, a in FP64 + the FP32 filter threshold), authoritative
-// FP64 best + index per (plane, slot), filtered min/argmin with leader updates and 128-bit
-// CAS merges of dirty positions.
+// per-warp rings (entries: df, dg, a in FP64 + the FP32 filter threshold).  The exact path
+// writes through: a row / column group leader merges its (value, index) into the global
+// merge key with a 128-bit CAS (lexicographic min, reading G2) and lowers the ring's
+// threshold; the authoritative bests live only in global memory, which keeps the ring at
+// 32 B per (position, dim) and the kernel at 8 resident warps per SM.
 #include "mp_diag.cuh"
 
 namespace mpk {
 
+// ring entry: the staged FP64 best (global key value) lands in (thr, pad) and fixup()
+// replaces it in place by the FP32 filter threshold
 struct alignas(16) E64 { double df, dg, a; float thr; unsigned pad; };
 
 template <int DL, int G> struct Smem64f {
     using Gm = Geo<G, 1>;
     static constexpr int D = DL * G;
     static constexpr size_t ring_bytes =
-        (((size_t)D * (Gm::PSR + Gm::PSC) * (sizeof(E64) + 8 + 4)) + 15) & ~(size_t)15;
-    static constexpr size_t flag_bytes = ((Gm::RING_R + Gm::RING_C) * 4 + 15) & ~(size_t)15;
-    static constexpr size_t bytes_per_warp = ring_bytes + flag_bytes + (size_t)DL * 32 * sizeof(double);
+        (((size_t)D * (Gm::PSR + Gm::PSC) * sizeof(E64)) + 15) & ~(size_t)15;
+    static constexpr size_t bytes_per_warp = ring_bytes;
     static constexpr int WPB = bytes_per_warp * 4 <= 112 * 1024 ? 4 : bytes_per_warp * 2 <= 112 * 1024 ? 2 : 1;
 };
 
@@ -52,13 +55,6 @@ mp_diag64f(const MainParams p) {
     unsigned char* wbase = smem_raw + (size_t)warp * SM::bytes_per_warp;
     E64* rowv = reinterpret_cast<E64*>(wbase);
     E64* colv = rowv + (size_t)D * PSR;
-    double* rowb = reinterpret_cast<double*>(colv + (size_t)D * PSC);
-    double* colb = rowb + (size_t)D * PSR;
-    unsigned* rowi = reinterpret_cast<unsigned*>(colb + (size_t)D * PSC);
-    unsigned* coli = rowi + (size_t)D * PSR;
-    unsigned* rowdirty = reinterpret_cast<unsigned*>(wbase + SM::ring_bytes);
-    unsigned* coldirty = rowdirty + Gm::RING_R;
-    double* ssc = reinterpret_cast<double*>(wbase + SM::ring_bytes + SM::flag_bytes);
 
     const double4* __restrict__ st_q = reinterpret_cast<const double4*>(p.st_q);
     const double4* __restrict__ st_r = reinterpret_cast<const double4*>(p.st_r);
@@ -72,7 +68,6 @@ mp_diag64f(const MainParams p) {
     const int d = p.d, m = p.m, H = p.H, HT = p.HT;
     const int n32 = (int)n;
     const double two_m = (double)(2 * m);
-    const float two_mf = (float)(2 * m);
     const double INF = PT<double>::inf();
     // filter margin: relative FP32 rounding of S_k (D^2 -> float, approx sqrt, k adds)
     const double margin = 1.0 + ldexp(1.0, -20) + (double)d * ldexp(1.0, -22);
@@ -89,9 +84,6 @@ mp_diag64f(const MainParams p) {
         const int cnt = p_hi - p_lo;
         if (cnt <= 0) return;
         E64* buf = is_row ? rowv : colv;
-        double* bb = is_row ? rowb : colb;
-        unsigned* ib = is_row ? rowi : coli;
-        unsigned* dflag = is_row ? rowdirty : coldirty;
         const int ps = is_row ? PSR : PSC;
         const double4* __restrict__ st = is_row ? st_q : st_r;
         const bool want_thr = is_row || SELF;
@@ -100,7 +92,6 @@ mp_diag64f(const MainParams p) {
             const int pos = base + p_lo + pi;
             if (pos < 0 || pos >= n32) continue;
             const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
-            if (pl == 0) dflag[sl] = 0;
             E64* dst = &buf[pl * ps + sl];
             if (pl < d) {
                 const double4* src = st + (size_t)pos * d + pl;
@@ -110,14 +101,8 @@ mp_diag64f(const MainParams p) {
                 dst->df = 0; dst->dg = 0; dst->a = INF;
             }
             const int rk = rank_of_plane<DL, G>(pl);
-            if (rk < d && want_thr) {
-                const K* kp = keys + (size_t)pos * d + rk;
-                cp_async8(&bb[pl * ps + sl], &kp->v);
-                cp_async4(&ib[pl * ps + sl], &kp->i);
-            } else {
-                bb[pl * ps + sl] = -INF;
-                ib[pl * ps + sl] = 0x7fffffffu;
-            }
+            if (rk < d && want_thr) cp_async8(&dst->thr, &keys[(size_t)pos * d + rk].v);
+            else *reinterpret_cast<double*>(&dst->thr) = -INF;  // never hit
         }
     };
     // FP32 filter thresholds from the landed FP64 bests (rounded up, widened by the margin)
@@ -125,43 +110,16 @@ mp_diag64f(const MainParams p) {
         const int cnt = p_hi - p_lo;
         if (cnt <= 0) return;
         E64* buf = is_row ? rowv : colv;
-        const double* bb = is_row ? rowb : colb;
         const int ps = is_row ? PSR : PSC;
         for (int e = lane; e < cnt * D; e += 32) {
             const int pi = e / D, pl = e - pi * D;
             const int pos = base + p_lo + pi;
             if (pos < 0 || pos >= n32) continue;
             const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
-            buf[pl * ps + sl].thr = __double2float_ru(bb[pl * ps + sl] * margin);
+            E64& en = buf[pl * ps + sl];
+            en.thr = __double2float_ru(*reinterpret_cast<const double*>(&en.thr) * margin);
         }
     };
-    auto evict = [&](bool is_row, int base, int p_lo, int p_hi) {
-        if (!is_row && !SELF) return;
-        const int cnt = p_hi - p_lo;
-        if (cnt <= 0) return;
-        const double* bb = is_row ? rowb : colb;
-        const unsigned* ib = is_row ? rowi : coli;
-        const unsigned* dflag = is_row ? rowdirty : coldirty;
-        const int ps = is_row ? PSR : PSC;
-        bool any = false;
-        for (int pi = lane; pi < cnt; pi += 32) {
-            const int pos = base + p_lo + pi;
-            if (pos >= 0 && pos < n32) any |= dflag[is_row ? Gm::srow(pos) : Gm::scol(pos)] != 0;
-        }
-        if (!__any_sync(FULL, any)) return;
-        for (int e = lane; e < cnt * D; e += 32) {
-            const int pi = e / D, pl = e - pi * D;
-            const int pos = base + p_lo + pi;
-            if (pos < 0 || pos >= n32) continue;
-            const int sl = is_row ? Gm::srow(pos) : Gm::scol(pos);
-            if (dflag[sl] == 0) continue;
-            const int rk = rank_of_plane<DL, G>(pl);
-            if (rk >= d) continue;
-            const unsigned ix = ib[pl * ps + sl];
-            if (ix & DIRTY) KO::merge(keys + (size_t)pos * d + rk, bb[pl * ps + sl], ix & ~DIRTY);
-        }
-    };
-
     for (;;) {
         long long t = 0;
         if (lane == 0) t = (long long)atomicAdd(p.counter, 1ull);
@@ -218,7 +176,7 @@ mp_diag64f(const MainParams p) {
         const int nrows = (int)(r1 - r0);
         const int s_end = nrows + CW * (RA - 1);
         const int R0 = (int)r0, C0 = (int)(r0 + delta0);
-        int row_in = min(SB, nrows), col_in = min(SB, s_end) + CW - 1, row_out = 0, col_out = 0;
+        int row_in = min(SB, nrows), col_in = min(SB, s_end) + CW - 1;
         int fx_r0 = 0, fx_c0 = 0;
         stage(true, R0, 0, row_in);
         stage(false, C0, 0, col_in);
@@ -298,31 +256,32 @@ mp_diag64f(const MainParams p) {
 #pragma unroll
                 for (int kk = 0; kk < DL; ++kk) S[kk] += excl;
             }
+            if (!active) {
 #pragma unroll
-            for (int kk = 0; kk < DL; ++kk) ssc[kk * 32 + lane] = active ? S[kk] : INF;
-            __syncwarp();
+                for (int kk = 0; kk < DL; ++kk) S[kk] = INF;
+            }
+            // Eq. (3), write-through: rank by rank (S rotates through S[0], so no dynamic
+            // register indexing), group min by shuffles, the lowest-index leader merges
+            // (value, index) into the global key and lowers the ring threshold
 #pragma unroll 1
             for (int kk = 0; kk < DL; ++kk) {
                 const int pl = kk * G + g;
-                const double v = ssc[kk * 32 + lane];
-                const bool need_r = __any_sync(FULL, v <= rowb[pl * PSR + sr]);
-                const bool need_c = SELF && __any_sync(FULL, v <= colb[pl * PSC + sc]);
+                const double v = S[0];
+#pragma unroll
+                for (int q = 0; q + 1 < DL; ++q) S[q] = S[q + 1];
+                const int rk = rank_of_plane<DL, G>(pl);
+                const bool need_r = __any_sync(FULL, v <= (double)rowv[pl * PSR + sr].thr);
+                const bool need_c = SELF && __any_sync(FULL, v <= (double)colv[pl * PSC + sc].thr);
                 if (!need_r && !need_c) continue;
                 double vr = v;
 #pragma unroll
                 for (int bit = 0; bit < Gm::LOG_CA; ++bit)
                     vr = PT<double>::vmin(vr, __shfl_xor_sync(FULL, vr, 1 << (bit + Gm::LOG_G)));
                 const unsigned eqr = __ballot_sync(FULL, v == vr) & gmask_row;
-                if (need_r && vr < INF && lane == __ffs(eqr) - 1) {
-                    const int ix = pl * PSR + sr;
-                    const double cur = rowb[ix];
-                    const unsigned ci = rowi[ix] & ~DIRTY;
-                    if (vr < cur || (vr == cur && (unsigned)col < ci)) {
-                        rowb[ix] = vr;
-                        rowi[ix] = (unsigned)col | DIRTY;
-                        rowv[ix].thr = __double2float_ru(vr * margin);
-                        rowdirty[sr] = 1;
-                    }
+                if (need_r && vr < INF && rk < d && lane == __ffs(eqr) - 1) {
+                    KO::merge(keys + (size_t)row * d + rk, vr, (unsigned)col);
+                    float& th = rowv[pl * PSR + sr].thr;
+                    th = fminf(th, __double2float_ru(vr * margin));
                 }
                 if (SELF && need_c) {
                     double vc = v;
@@ -330,16 +289,10 @@ mp_diag64f(const MainParams p) {
                     for (int bit = 0; bit < 5 - Gm::LOG_G - Gm::LOG_CA; ++bit)
                         vc = PT<double>::vmin(vc, __shfl_xor_sync(FULL, vc, 1 << (bit + Gm::LOG_G + Gm::LOG_CA)));
                     const unsigned eqc = __ballot_sync(FULL, v == vc) & gmask_col;
-                    if (vc < INF && eqc != 0 && lane == 31 - __clz(eqc)) {
-                        const int ix = pl * PSC + sc;
-                        const double cur = colb[ix];
-                        const unsigned ci = coli[ix] & ~DIRTY;
-                        if (vc < cur || (vc == cur && (unsigned)row < ci)) {
-                            colb[ix] = vc;
-                            coli[ix] = (unsigned)row | DIRTY;
-                            colv[ix].thr = __double2float_ru(vc * margin);
-                            coldirty[sc] = 1;
-                        }
+                    if (vc < INF && rk < d && eqc != 0 && lane == 31 - __clz(eqc)) {
+                        KO::merge(keys + (size_t)col * d + rk, vc, (unsigned)row);
+                        float& th = colv[pl * PSC + sc].thr;
+                        th = fminf(th, __double2float_ru(vc * margin));
                     }
                 }
             }
@@ -355,11 +308,6 @@ mp_diag64f(const MainParams p) {
                 else if (row > lo && row < hi) seed_cell(row);
                 seeded_step = s0 == 0 ? -1 : s0;
             }
-            const int rx = min(max(s0 - CW * (RA - 1), 0), nrows);
-            evict(true, R0, row_out, rx);
-            row_out = rx;
-            evict(false, C0, col_out, s0);
-            col_out = s0;
             const int nxt = min(s0 + 2 * SB, s_end);
             const int r_need = min(nxt, nrows), c_need = nxt + CW - 1;
             stage(true, R0, row_in, r_need);
@@ -378,8 +326,6 @@ mp_diag64f(const MainParams p) {
             fx_c0 = col_in;
             __syncwarp();
         }
-        evict(true, R0, row_out, nrows);
-        evict(false, C0, col_out, col_in);
         __syncwarp();
     }
 }
