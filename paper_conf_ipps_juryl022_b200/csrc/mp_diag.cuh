@@ -576,7 +576,7 @@ mp_diag(const MainParams p) {
 
             // thresholds stay in registers for small per-lane dim counts; wide lanes
             // re-read them from the ring after the sort (register budget)
-            constexpr bool KEEP = (DL <= MP_KEEP_DL);
+            constexpr bool KEEP = (DL * W <= MP_KEEP_DL);
             T S[W][DL], tr[KEEP ? DL : 1], tc0[KEEP ? DL : 1];
 #pragma unroll
             for (int kk = 0; kk < DL; ++kk) {

@@ -21,6 +21,8 @@
 
 namespace mpk {
 
+struct PendM { double v; unsigned long long key; unsigned idx, pad; };
+
 // ring entry: the staged FP64 best (global key value) lands in (thr, pad) and fixup()
 // replaces it in place by the FP32 filter threshold
 struct alignas(16) E64 { double df, dg, a; float thr; unsigned pad; };
@@ -30,7 +32,9 @@ template <int DL, int G> struct Smem64f {
     static constexpr int D = DL * G;
     static constexpr size_t ring_bytes =
         (((size_t)D * (Gm::PSR + Gm::PSC) * sizeof(E64)) + 15) & ~(size_t)15;
-    static constexpr size_t bytes_per_warp = ring_bytes;
+    // pending write-through merges (key slot, value, index), flushed by all lanes at once
+    static constexpr int QN = 64;
+    static constexpr size_t bytes_per_warp = ring_bytes + QN * sizeof(PendM);
     static constexpr int WPB = bytes_per_warp * 4 <= 112 * 1024 ? 4 : bytes_per_warp * 2 <= 112 * 1024 ? 2 : 1;
 };
 
@@ -53,6 +57,8 @@ mp_diag64f(const MainParams p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     unsigned char* wbase = smem_raw + (size_t)warp * SM::bytes_per_warp;
+    PendM* pend = reinterpret_cast<PendM*>(wbase + SM::ring_bytes);
+    int npend = 0;  // warp-uniform
     E64* rowv = reinterpret_cast<E64*>(wbase);
     E64* colv = rowv + (size_t)D * PSR;
 
@@ -120,6 +126,15 @@ mp_diag64f(const MainParams p) {
             en.thr = __double2float_ru(*reinterpret_cast<const double*>(&en.thr) * margin);
         }
     };
+    // merge the pending (value, index) pairs into the global keys: one CAS loop per lane, so
+    // the L2 round trips of a batch overlap instead of serialising behind single leaders
+    auto flush = [&]() {
+        __syncwarp();
+        for (int q = lane; q < npend; q += 32) KO::merge(keys + pend[q].key, pend[q].v, pend[q].idx);
+        npend = 0;
+        __syncwarp();
+    };
+
     for (;;) {
         long long t = 0;
         if (lane == 0) t = (long long)atomicAdd(p.counter, 1ull);
@@ -273,27 +288,40 @@ mp_diag64f(const MainParams p) {
                 const bool need_r = __any_sync(FULL, v <= (double)rowv[pl * PSR + sr].thr);
                 const bool need_c = SELF && __any_sync(FULL, v <= (double)colv[pl * PSC + sc].thr);
                 if (!need_r && !need_c) continue;
+                if (npend > SM::QN - 32) flush();  // room for one round of leaders
                 double vr = v;
 #pragma unroll
                 for (int bit = 0; bit < Gm::LOG_CA; ++bit)
                     vr = PT<double>::vmin(vr, __shfl_xor_sync(FULL, vr, 1 << (bit + Gm::LOG_G)));
                 const unsigned eqr = __ballot_sync(FULL, v == vr) & gmask_row;
-                if (need_r && vr < INF && rk < d && lane == __ffs(eqr) - 1) {
-                    KO::merge(keys + (size_t)row * d + rk, vr, (unsigned)col);
+                const bool lead_r = need_r && vr < INF && rk < d && lane == __ffs(eqr) - 1;
+                const unsigned lr = __ballot_sync(FULL, lead_r);
+                if (lead_r) {
+                    PendM& e = pend[npend + __popc(lr & ((1u << lane) - 1))];
+                    e.v = vr;
+                    e.key = (unsigned long long)row * d + rk;
+                    e.idx = (unsigned)col;
                     float& th = rowv[pl * PSR + sr].thr;
                     th = fminf(th, __double2float_ru(vr * margin));
                 }
+                npend += __popc(lr);
                 if (SELF && need_c) {
                     double vc = v;
 #pragma unroll
                     for (int bit = 0; bit < 5 - Gm::LOG_G - Gm::LOG_CA; ++bit)
                         vc = PT<double>::vmin(vc, __shfl_xor_sync(FULL, vc, 1 << (bit + Gm::LOG_G + Gm::LOG_CA)));
                     const unsigned eqc = __ballot_sync(FULL, v == vc) & gmask_col;
-                    if (vc < INF && rk < d && eqc != 0 && lane == 31 - __clz(eqc)) {
-                        KO::merge(keys + (size_t)col * d + rk, vc, (unsigned)row);
+                    const bool lead_c = vc < INF && rk < d && eqc != 0 && lane == 31 - __clz(eqc);
+                    const unsigned lcm = __ballot_sync(FULL, lead_c);
+                    if (lead_c) {
+                        PendM& e = pend[npend + __popc(lcm & ((1u << lane) - 1))];
+                        e.v = vc;
+                        e.key = (unsigned long long)col * d + rk;
+                        e.idx = (unsigned)row;
                         float& th = colv[pl * PSC + sc].thr;
                         th = fminf(th, __double2float_ru(vc * margin));
                     }
+                    npend += __popc(lcm);
                 }
             }
             __syncwarp();
@@ -318,6 +346,7 @@ mp_diag64f(const MainParams p) {
             const int s1 = min(s0 + SB, s_end);
 #pragma unroll 1
             for (int ss = s0; ss < s1; ++ss) step(ss);
+            if (npend) flush();
             cp_async_wait_all();
             __syncwarp();
             fixup(true, R0, fx_r0, row_in);
