@@ -146,6 +146,47 @@ def load_peaks():
         return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "sm_max_mhz": NOMINAL_SM_MHZ}, "fallback"
 
 
+def alu_ops_mode(d: int, self_join: bool, prec: str) -> float:
+    """ALU-pipe ops per computed cell*dim by precision mode: FP32 and FP64 (whose common path is
+    the FP32 filter: same sort, scan and compares) as alu_ops_per_cell_dim; FP16 / Mixed pack two
+    cells in a half2, so each HMNMX2 / HSETP2 serves two cell*dims."""
+    ops = alu_ops_per_cell_dim(d, self_join)
+    return ops / 2.0 if prec in ("fp16", "mixed", "fp16c") else ops
+
+
+def band_probe(ctx, torch, dev, name: str, prec: str, target_cell_dims: float = 3e11):
+    """Throughput of one diagonal band of a larger BASELINE config at its full input size: the
+    unit one rank computes under bench.py --gpus N (mp_partial_device), timed by the library's
+    CUDA events around the main kernel.  The band is the middle one of a W-way equal-cell split
+    sized to ~target_cell_dims computed cell*dims, so the probe takes seconds, not the minutes
+    to hours of the full grid on one GPU."""
+    from paper_conf_ipps_juryl022_b200 import mstamp
+    cfg = datagen.make(name)
+    d, n, m, e = cfg["d"], cfg["n"], cfg["m"], cfg["exclusion"]
+    self_join = cfg["Tr"] is None
+    total = computed_cells(n, e, self_join) * d
+    W = max(1, int(round(total / target_cell_dims)))
+    r = W // 2
+    _, bc = mstamp.plan_bands(d, n, m, prec, e, self_join, W)
+    T = torch.from_numpy(cfg["T"]).to(dev)
+    Tr = None if self_join else torch.from_numpy(cfg["Tr"]).to(dev)
+    keys = torch.empty(mstamp.key_words(d, n, prec), dtype=torch.int64, device=dev)
+    kms = []
+    for _ in range(2):  # the first launch also pays one-time setup; report the second
+        ctx.partial_device(T, m, keys, r, W, prec, e, Tr=Tr)
+        torch.cuda.synchronize()
+        kms.append(ctx.last_timing()[0])
+    del T, Tr, keys
+    torch.cuda.empty_cache()
+    cd = int(bc[r]) * d
+    rate = cd / (kms[-1] * 1e-3)
+    peak = SM_COUNT * ALU_LANES * NOMINAL_SM_MHZ * 1e6
+    return {"workload": f"{'self' if self_join else 'AB'}-join d={d} n={n} m={m}", "precision": prec,
+            "band": [r, W], "band_cell_dims": cd, "main_kernel_ms": kms[-1],
+            "computed_cell_dims_per_s": rate, "alu_frac": rate * alu_ops_mode(d, self_join, prec) / peak,
+            "full_grid_estimate_s_1gpu": total / rate}
+
+
 def launches_per_step(prec: str, self_join: bool) -> int:
     # check_finite (1 per series) + precompute (pre_stats, pre_diff, pre_pm) per series
     # + init_keys + mp_diag + [keys64_to_ext] + finalize
@@ -226,6 +267,8 @@ def main():
     ap.add_argument("--ref-seconds", type=float, default=15.0)
     ap.add_argument("--no-per-precision", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-per-config", action="store_true",
+                    help="skip the one-band throughput probes of the larger BASELINE configs")
     ap.add_argument("--backend", default="nccl", help="process-group backend for N>1 (gloo: functional "
                     "test of the multi-rank path, e.g. several ranks on one GPU via MP_BENCH_DEVICE)")
     args = ap.parse_args()
@@ -309,6 +352,15 @@ def main():
                 continue
             p_ms, p_kms, _ = timed(prec, max(1, min(args.steps, 3)), 1)
             per_prec[prec] = {"value": dn2 / (p_ms * 1e-3), "ms_per_step": p_ms, "main_kernel_ms": p_kms}
+        cells0 = computed_cells(n, e, self_join)
+        for prec, v in per_prec.items():  # ALU roofline fraction of the main kernel per mode
+            rate = cells0 * d / (v["main_kernel_ms"] * 1e-3)
+            v["alu_frac"] = rate * alu_ops_mode(d, self_join, prec) / (SM_COUNT * ALU_LANES * NOMINAL_SM_MHZ * 1e6)
+
+    per_cfg = {}
+    if not args.no_per_config and world == 1:
+        for name, prec in (("C3", "fp32"), ("C3", "mixed"), ("C4", "fp32"), ("C5", "fp32")):
+            per_cfg[f"{name}/{prec}"] = band_probe(ctx, torch, dev, name, prec)
 
     # e2e through the C-ABI host entry point (pinned host buffers, H2D + D2H inside)
     e2e = None
@@ -357,7 +409,7 @@ def main():
                 "vs_baseline": None, "dtype": {"fp64": "f64", "fp32": "f32"}.get(args.precision, args.precision),
                 "data": "synthetic", "config": config_json(args, cfg), "roofline": roof, "cpu_baseline": cpu,
                 "e2e": e2e, "gpu_launches": launches_per_step(args.precision, self_join) * args.steps,
-                "clocks": clocks, "per_precision": per_prec,
+                "clocks": clocks, "per_precision": per_prec, "per_config_band": per_cfg or None,
                 "computed_cells_per_s": cells * d / (ms * 1e-3)}
         print(json.dumps(line), flush=True)
     ctx.close()
