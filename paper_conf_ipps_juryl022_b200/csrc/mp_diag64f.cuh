@@ -288,12 +288,12 @@ mp_diag64f(const MainParams p) {
                 const bool need_r = __any_sync(FULL, v <= (double)rowv[pl * PSR + sr].thr);
                 const bool need_c = SELF && __any_sync(FULL, v <= (double)colv[pl * PSC + sc].thr);
                 if (!need_r && !need_c) continue;
-                if (npend > SM::QN - 32) flush();  // room for one round of leaders
                 double vr = v;
 #pragma unroll
                 for (int bit = 0; bit < Gm::LOG_CA; ++bit)
                     vr = PT<double>::vmin(vr, __shfl_xor_sync(FULL, vr, 1 << (bit + Gm::LOG_G)));
                 const unsigned eqr = __ballot_sync(FULL, v == vr) & gmask_row;
+                if (npend > SM::QN - 32) flush();  // room for one round of leaders (<= 32)
                 const bool lead_r = need_r && vr < INF && rk < d && lane == __ffs(eqr) - 1;
                 const unsigned lr = __ballot_sync(FULL, lead_r);
                 if (lead_r) {
@@ -311,6 +311,7 @@ mp_diag64f(const MainParams p) {
                     for (int bit = 0; bit < 5 - Gm::LOG_G - Gm::LOG_CA; ++bit)
                         vc = PT<double>::vmin(vc, __shfl_xor_sync(FULL, vc, 1 << (bit + Gm::LOG_G + Gm::LOG_CA)));
                     const unsigned eqc = __ballot_sync(FULL, v == vc) & gmask_col;
+                    if (npend > SM::QN - 32) flush();
                     const bool lead_c = vc < INF && rk < d && eqc != 0 && lane == 31 - __clz(eqc);
                     const unsigned lcm = __ballot_sync(FULL, lead_c);
                     if (lead_c) {

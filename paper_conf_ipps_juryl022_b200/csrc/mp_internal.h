@@ -47,7 +47,7 @@ struct PreParams {
 enum { P64 = 0, P32 = 1, P16 = 2, PMIX = 3, P16C = 4 };
 
 // Variant selection for a given (precision, d): dims per lane DL and lanes per cell G.
-struct Variant { int DL; int G; int W; int NC; };
+struct Variant { int DL; int G; int W; int NC; int cta = 0; /* warps per block of the block-cooperative kernel, 0: warp tiles */ };
 Variant pick_variant(int prec, int d);
 size_t smem_per_block(int prec, int d, bool self);
 int variant_warps_per_block(int prec, int d, bool self);

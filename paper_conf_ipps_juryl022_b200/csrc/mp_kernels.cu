@@ -3,6 +3,7 @@
 // the heavy template variants compile in parallel).
 #include "mp_diag16.cuh"
 #include "mp_diag64f.cuh"
+#include "mp_diag_cta.cuh"
 
 namespace mpk {
 
@@ -329,10 +330,10 @@ Variant pick_variant(int prec, int d) {
     } else {
         if (dp <= 8) { v.DL = dp; v.G = 1; v.W = 2; }
         else if (dp == 16) { v.DL = 16; v.G = 1; v.W = 1; }
-        else if (dp <= 512) { v.DL = 16; v.G = dp / 16; v.W = 1; }
+        else if (dp <= 512) { v.DL = 16; v.G = dp / 16; v.W = 1; if (MP_CTA_NW && dp >= 64) v.cta = MP_CTA_NW; }
         else { v.DL = 32; v.G = dp / 32; v.W = 1; }
     }
-    v.NC = 32 / v.G * v.W;
+    v.NC = v.cta ? 32 * v.cta / v.G : 32 / v.G * v.W;
     return v;
 }
 
@@ -384,8 +385,26 @@ static long long dispatch_64f(int op, int DL, int G, const MainParams* p, int gr
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
 }
 
+template <bool SELF>
+static long long dispatch_cta(int op, int G, const MainParams* p, int grid, cudaStream_t s) {
+#define MP_CCASE(g)                                                                        \
+    if (G == g) {                                                                          \
+        using I = InstCta<16, g, MP_CTA_NW, SELF>;                                         \
+        if (op == 0) return (long long)I::smem();                                          \
+        if (op == 1) return (long long)I::launch(*p, grid, s);                             \
+        if (op == 3) return 1;  /* one tile per block */                                   \
+        return I::blocks_per_sm();                                                         \
+    }
+#if MP_CTA_NW
+    MP_CCASE(4) MP_CCASE(8) MP_CCASE(16) MP_CCASE(32)
+#endif
+#undef MP_CCASE
+    return op == 1 ? (long long)cudaErrorInvalidValue : 0;
+}
+
 static long long dispatch(int op, int prec, bool self, int d, const MainParams* p, int grid, cudaStream_t s) {
     const Variant v = pick_variant(prec, d);
+    if (v.cta) return self ? dispatch_cta<true>(op, v.G, p, grid, s) : dispatch_cta<false>(op, v.G, p, grid, s);
     if (prec == P16) return self ? dispatch_h<true, 0>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 0>(op, v.DL, v.G, p, grid, s);
     if (prec == PMIX) return self ? dispatch_h<true, 1>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 1>(op, v.DL, v.G, p, grid, s);
     if (prec == P16C) return self ? dispatch_h<true, 2>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 2>(op, v.DL, v.G, p, grid, s);

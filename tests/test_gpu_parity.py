@@ -48,6 +48,8 @@ SHAPES = [  # (d, n, m, exclusion, seed): ragged tails, several tiles, odd d, ti
     (1, 300, 8, 2, 1), (2, 77, 5, 1, 2), (3, 1500, 16, 4, 3), (5, 700, 32, 8, 4),
     (8, 2100, 12, 3, 5), (16, 1100, 64, 16, 6), (17, 600, 16, 4, 7), (32, 400, 8, 2, 8),
     (33, 300, 10, 3, 9), (64, 250, 16, 4, 10), (100, 200, 8, 2, 11), (7, 5000, 24, 6, 12),
+    # large d (block-cooperative FP32 kernel: G = 4 / 8 / 16 / 32 lanes per cell), several tiles
+    (64, 2500, 32, 8, 13), (130, 400, 12, 3, 14), (256, 300, 16, 4, 15), (300, 150, 8, 2, 16),
 ]
 
 
@@ -64,7 +66,8 @@ def test_random_shapes_self(ctx, oracle_mod, prec, shape):
 
 
 @pytest.mark.parametrize("prec", ["fp64", "fp32"])
-@pytest.mark.parametrize("shape", [(1, 200, 8, 21), (4, 900, 16, 22), (16, 500, 32, 23), (40, 150, 8, 24)])
+@pytest.mark.parametrize("shape", [(1, 200, 8, 21), (4, 900, 16, 22), (16, 500, 32, 23), (40, 150, 8, 24),
+                                   (128, 600, 16, 25), (256, 200, 8, 26)])
 def test_random_shapes_ab(ctx, oracle_mod, prec, shape):
     d, n, m, seed = shape
     Tq, Tr = datagen.random_walk_ab(d, n, m, seed)
