@@ -21,6 +21,9 @@
 // when they leave the ring.
 #include "mp_diag.cuh"
 
+#ifndef MP_CTA_SB
+#define MP_CTA_SB 1   // steps per staging batch (one block barrier per batch)
+#endif
 #ifndef MP_CTA_NW
 #define MP_CTA_NW 4   // warps per block of the block-cooperative large-d FP32 kernel (0: off)
 #endif
@@ -31,7 +34,7 @@ template <int DL, int G, int NW> struct CtaGeo {
     static constexpr int NT = 32 * NW;             // threads per block
     static constexpr int NCC = NT / G;             // cells (diagonals) per block tile
     static constexpr int D = DL * G;
-    static constexpr int SB = 1;                   // steps per staging batch
+    static constexpr int SB = MP_CTA_SB;           // steps per staging batch
     // ring slots: positions of the current batch, the prefetched next one and the batch being
     // evicted stay distinct, so eviction reads and prefetch writes never touch the same slot
     static constexpr int RR = 3 * SB;
