@@ -655,9 +655,28 @@ mp_diag(const MainParams p) {
 #pragma unroll
                     for (int kk = 0; kk < DL; ++kk) ssc[(u * DL + kk) * 32 + lane] = active[u] ? S[u][kk] : INF;
                 __syncwarp();
+                // ranks some lane can improve (compared with the current ring bests, from
+                // shared memory so no register stays live across the slow path): one warp OR,
+                // then the loop visits only those ranks -- a slow step touches 1-2 of DL ranks
+                unsigned rk_bits = 0;
+#pragma unroll
+                for (int kk = 0; kk < DL; ++kk) {
+                    const int pl = kk * G + g;
+                    const T tr_k = rowv[pl * PSR + sr].w;
+                    bool hk = false;
+#pragma unroll
+                    for (int u = 0; u < W; ++u) {
+                        const T v = ssc[(u * DL + kk) * 32 + lane];
+                        hk |= v <= tr_k;
+                        if (SELF) hk |= v <= colv[pl * PSC + Gm::scol(col[u])].w;
+                    }
+                    rk_bits |= (unsigned)hk << kk;
+                }
+                rk_bits = __reduce_or_sync(FULL, rk_bits);
                 DMask mark_r = 0, mark_c = 0;  // ring slots this lane's leader updates dirtied
 #pragma unroll 1
-                for (int kk = 0; kk < DL; ++kk) {
+                for (; rk_bits != 0; rk_bits &= rk_bits - 1) {
+                    const int kk = __ffs(rk_bits) - 1;
                     const int pl = kk * G + g;
                     T v[W];
 #pragma unroll

@@ -73,6 +73,97 @@ __device__ __forceinline__ void ldv(const T* __restrict__ rowp, int g, T (&out)[
     }
 }
 
+// Seeds of one cell pair (diagonals delta0, delta0 + 1): direct centred dot products
+// (reading G8) at rows row0 / row1 (cells with ok_u false keep their QT).
+// Mixed -> FP32 operands and accumulation rounded to half (the FP32 precalc); FP16 -> half
+// arithmetic; FP16C -> half arithmetic with Kahan compensation.  When both cells start on the
+// same row the row window is shared and the second column window is the first shifted by one.
+template <int DL, int G, int MODE, class TS>
+__device__ __forceinline__ void seed_pair_h(const TS* __restrict__ tw_q, const TS* __restrict__ tw_r,
+                                            const TS* __restrict__ mu_q, const TS* __restrict__ mu_r,
+                                            int m, int d, int g, long long delta0, bool ok0, bool ok1,
+                                            long long row0, long long row1, __half2 (&QT)[DL]) {
+    constexpr int D = DL * G;
+    const long long delta[2] = {delta0, delta0 + 1};
+    using TA = TS;
+    const bool same = ok0 && ok1 && row0 == row1;
+    TA acc0[DL], acc1[DL];
+#pragma unroll
+    for (int kk = 0; kk < DL; ++kk) { acc0[kk] = (TA)0.f; acc1[kk] = (TA)0.f; }
+    auto kadd = [](TA& acc, TA& cp, TA v) {
+        if constexpr (MODE == 2) {  // compensated half accumulation
+            const TA y = v - cp;
+            const TA t2 = acc + y;
+            cp = (t2 - acc) - y;
+            acc = t2;
+        } else {
+            acc = acc + v;
+        }
+    };
+    // dims in chunks of one 16-byte vector per operand: the m-long loop keeps few
+    // operand registers live, so seeding does not set the kernel's register peak
+    constexpr int SC = (16 / (int)sizeof(TA)) < DL ? (16 / (int)sizeof(TA)) : DL;
+    if (same) {
+        const long long i0 = row0, j0 = row0 + delta[0];
+#pragma unroll
+        for (int c0 = 0; c0 < DL; c0 += SC) {
+            TA mq[SC], mr0[SC], mr1[SC], xr[SC], a0[SC], a1[SC], k0[SC], k1[SC];
+            ldv<TA, SC, G>(mu_q + i0 * D + c0 * G, g, mq);
+            ldv<TA, SC, G>(mu_r + j0 * D + c0 * G, g, mr0);
+            ldv<TA, SC, G>(mu_r + (j0 + 1) * D + c0 * G, g, mr1);
+            ldv<TA, SC, G>(tw_r + j0 * D + c0 * G, g, xr);
+#pragma unroll
+            for (int kk = 0; kk < SC; ++kk) { a0[kk] = (TA)0.f; a1[kk] = (TA)0.f; k0[kk] = (TA)0.f; k1[kk] = (TA)0.f; }
+#pragma unroll 4
+            for (int tt = 0; tt < m; ++tt) {
+                TA xq[SC], xn[SC];
+                ldv<TA, SC, G>(tw_q + (i0 + tt) * D + c0 * G, g, xq);
+                ldv<TA, SC, G>(tw_r + (j0 + tt + 1) * D + c0 * G, g, xn);   // j0 + m <= L - 1 (cell 1 valid)
+#pragma unroll
+                for (int kk = 0; kk < SC; ++kk) {
+                    const TA cq = xq[kk] - mq[kk];
+                    kadd(a0[kk], k0[kk], cq * (xr[kk] - mr0[kk]));
+                    kadd(a1[kk], k1[kk], cq * (xn[kk] - mr1[kk]));
+                    xr[kk] = xn[kk];
+                }
+            }
+#pragma unroll
+            for (int kk = 0; kk < SC; ++kk) { acc0[c0 + kk] = a0[kk]; acc1[c0 + kk] = a1[kk]; }
+        }
+    } else {
+#pragma unroll 1
+        for (int u = 0; u < 2; ++u) {
+            if (!(u == 0 ? ok0 : ok1)) continue;
+            const long long i0 = u == 0 ? row0 : row1, j0 = i0 + delta[u];
+#pragma unroll
+            for (int c0 = 0; c0 < DL; c0 += SC) {
+                TA mq[SC], mr[SC], acc[SC], cp[SC];
+                ldv<TA, SC, G>(mu_q + i0 * D + c0 * G, g, mq);
+                ldv<TA, SC, G>(mu_r + j0 * D + c0 * G, g, mr);
+#pragma unroll
+                for (int kk = 0; kk < SC; ++kk) { acc[kk] = (TA)0.f; cp[kk] = (TA)0.f; }
+#pragma unroll 4
+                for (int tt = 0; tt < m; ++tt) {
+                    TA xq[SC], xr[SC];
+                    ldv<TA, SC, G>(tw_q + (i0 + tt) * D + c0 * G, g, xq);
+                    ldv<TA, SC, G>(tw_r + (j0 + tt) * D + c0 * G, g, xr);
+#pragma unroll
+                    for (int kk = 0; kk < SC; ++kk) kadd(acc[kk], cp[kk], (xq[kk] - mq[kk]) * (xr[kk] - mr[kk]));
+                }
+#pragma unroll
+                for (int kk = 0; kk < SC; ++kk) { if (u == 0) acc0[c0 + kk] = acc[kk]; else acc1[c0 + kk] = acc[kk]; }
+            }
+        }
+    }
+#pragma unroll
+    for (int kk = 0; kk < DL; ++kk) {
+        const bool pad = (kk * G + g) >= d;
+        const __half h0 = __float2half_rn(pad ? -1.f : (float)acc0[kk]);
+        const __half h1 = __float2half_rn(pad ? -1.f : (float)acc1[kk]);
+        QT[kk] = __halves2half2(ok0 ? h0 : __low2half(QT[kk]), ok1 ? h1 : __high2half(QT[kk]));
+    }
+}
+
 // MODE: 0 = FP16, 1 = Mixed (FP32 precalc and seeds), 2 = FP16C (half precalc and seeds with
 // Kahan-compensated sums, reading G17)
 template <int DL, int G, bool SELF, int MODE>
@@ -205,77 +296,9 @@ mp_diag_h(const MainParams p) {
             dlt[u] = (int)delta[u]; lo32[u] = (int)lo[u]; hi32[u] = (int)hi[u];
         }
 
-        // seeds (at the pair's first rows, then every H rows at warp-uniform steps): direct
-        // centred dot products (reading G8).  Mixed -> FP32 operands and
-        // accumulation rounded to half (the FP32 precalc); FP16 -> half arithmetic; FP16C ->
-        // half arithmetic with Kahan compensation.  When both cells start on the same row the
-        // row window is shared and the second column window is the first shifted by one.
         __half2 QT[DL];
         auto seed_pair = [&](bool ok0, bool ok1, long long row0, long long row1) {
-            using TA = TS;
-            const bool same = ok0 && ok1 && row0 == row1;
-            TA acc0[DL], acc1[DL], cp0[DL], cp1[DL];
-#pragma unroll
-            for (int kk = 0; kk < DL; ++kk) { acc0[kk] = (TA)0.f; acc1[kk] = (TA)0.f; cp0[kk] = (TA)0.f; cp1[kk] = (TA)0.f; }
-            auto kadd = [](TA& acc, TA& cp, TA v) {
-                if constexpr (MODE == 2) {  // compensated half accumulation
-                    const TA y = v - cp;
-                    const TA t2 = acc + y;
-                    cp = (t2 - acc) - y;
-                    acc = t2;
-                } else {
-                    acc = acc + v;
-                }
-            };
-            if (same) {
-                const long long i0 = row0, j0 = row0 + delta[0];
-                TA mq[DL], mr0[DL], mr1[DL], xr[DL];
-                ldv<TA, DL, G>(mu_q + i0 * D, g, mq);
-                ldv<TA, DL, G>(mu_r + j0 * D, g, mr0);
-                ldv<TA, DL, G>(mu_r + (j0 + 1) * D, g, mr1);
-                ldv<TA, DL, G>(tw_r + j0 * D, g, xr);
-#pragma unroll 2
-                for (int tt = 0; tt < m; ++tt) {
-                    TA xq[DL], xn[DL];
-                    ldv<TA, DL, G>(tw_q + (i0 + tt) * D, g, xq);
-                    ldv<TA, DL, G>(tw_r + (j0 + tt + 1) * D, g, xn);   // j0 + m <= L - 1 (cell 1 valid)
-#pragma unroll
-                    for (int kk = 0; kk < DL; ++kk) {
-                        const TA cq = xq[kk] - mq[kk];
-                        kadd(acc0[kk], cp0[kk], cq * (xr[kk] - mr0[kk]));
-                        kadd(acc1[kk], cp1[kk], cq * (xn[kk] - mr1[kk]));
-                        xr[kk] = xn[kk];
-                    }
-                }
-            } else {
-#pragma unroll 1
-                for (int u = 0; u < 2; ++u) {
-                    if (!(u == 0 ? ok0 : ok1)) continue;
-                    const long long i0 = u == 0 ? row0 : row1, j0 = i0 + delta[u];
-                    TA mq[DL], mr[DL], acc[DL], cp[DL];
-                    ldv<TA, DL, G>(mu_q + i0 * D, g, mq);
-                    ldv<TA, DL, G>(mu_r + j0 * D, g, mr);
-#pragma unroll
-                    for (int kk = 0; kk < DL; ++kk) { acc[kk] = (TA)0.f; cp[kk] = (TA)0.f; }
-#pragma unroll 2
-                    for (int tt = 0; tt < m; ++tt) {
-                        TA xq[DL], xr[DL];
-                        ldv<TA, DL, G>(tw_q + (i0 + tt) * D, g, xq);
-                        ldv<TA, DL, G>(tw_r + (j0 + tt) * D, g, xr);
-#pragma unroll
-                        for (int kk = 0; kk < DL; ++kk) kadd(acc[kk], cp[kk], (xq[kk] - mq[kk]) * (xr[kk] - mr[kk]));
-                    }
-#pragma unroll
-                    for (int kk = 0; kk < DL; ++kk) { if (u == 0) acc0[kk] = acc[kk]; else acc1[kk] = acc[kk]; }
-                }
-            }
-#pragma unroll
-            for (int kk = 0; kk < DL; ++kk) {
-                const bool pad = (kk * G + g) >= d;
-                const __half h0 = __float2half_rn(pad ? -1.f : (float)acc0[kk]);
-                const __half h1 = __float2half_rn(pad ? -1.f : (float)acc1[kk]);
-                QT[kk] = __halves2half2(ok0 ? h0 : __low2half(QT[kk]), ok1 ? h1 : __high2half(QT[kk]));
-            }
+            seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, delta[0], ok0, ok1, row0, row1, QT);
         };
 #pragma unroll
         for (int kk = 0; kk < DL; ++kk) QT[kk] = __float2half2_rn((kk * G + g) >= d ? -1.f : 0.f);
@@ -335,8 +358,19 @@ mp_diag_h(const MainParams p) {
             }
             sort_net<__half2, DL>(S);                                              // Eq. (2)
             if (G > 1) lane_merge<__half2, DL, G>(S, g);
+            // Eq. (2) inclusive scan, two independent half chains joined at the end (shorter
+            // dependency chain; the summation order differs only by rounding)
+            if constexpr (DL >= 8) {
 #pragma unroll
-            for (int kk = 1; kk < DL; ++kk) S[kk] = __hadd2(S[kk], S[kk - 1]);     // Eq. (2)
+                for (int kk = 1; kk < DL / 2; ++kk) S[kk] = __hadd2(S[kk], S[kk - 1]);
+#pragma unroll
+                for (int kk = DL / 2 + 1; kk < DL; ++kk) S[kk] = __hadd2(S[kk], S[kk - 1]);
+#pragma unroll
+                for (int kk = DL / 2; kk < DL; ++kk) S[kk] = __hadd2(S[kk], S[DL / 2 - 1]);
+            } else {
+#pragma unroll
+                for (int kk = 1; kk < DL; ++kk) S[kk] = __hadd2(S[kk], S[kk - 1]);
+            }
             if (G > 1) {
                 __half2 tot = S[DL - 1];
 #pragma unroll
@@ -365,9 +399,17 @@ mp_diag_h(const MainParams p) {
                     if (!active[1]) v = __halves2half2(__low2half(v), HINF);
                     ssc[kk * 32 + lane] = v;
                 }
+                // ranks some lane can improve (a superset: staged thresholds only decrease);
+                // the loop then visits only those -- a slow step typically touches 1-2 ranks
+                const unsigned act = (active[0] ? 0x0000ffffu : 0u) | (active[1] ? 0xffff0000u : 0u);
+                unsigned rk_bits = 0;
+#pragma unroll
+                for (int kk = 0; kk < DL; ++kk) rk_bits |= (unsigned)((__hle2_mask(S[kk], th[kk]) & act) != 0u) << kk;
+                rk_bits = __reduce_or_sync(FULL, rk_bits);
                 __syncwarp();
 #pragma unroll 1
-                for (int kk = 0; kk < DL; ++kk) {
+                for (; rk_bits != 0; rk_bits &= rk_bits - 1) {
+                    const int kk = __ffs(rk_bits) - 1;
                     const int pl = kk * G + g;
                     const int rk = g * DL + kk;  // rank held in register kk after the merge
                     const __half2 vh = ssc[kk * 32 + lane];

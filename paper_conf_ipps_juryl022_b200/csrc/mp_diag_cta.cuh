@@ -24,6 +24,9 @@
 #ifndef MP_CTA_SB
 #define MP_CTA_SB 1   // steps per staging batch (one block barrier per batch)
 #endif
+#ifndef MP_CTA_MIN_DP
+#define MP_CTA_MIN_DP 64   // smallest padded d that takes the block-cooperative kernel
+#endif
 #ifndef MP_CTA_NW
 #define MP_CTA_NW 4   // warps per block of the block-cooperative large-d FP32 kernel (0: off)
 #endif

@@ -4,6 +4,7 @@
 #include "mp_diag16.cuh"
 #include "mp_diag64f.cuh"
 #include "mp_diag_cta.cuh"
+#include "mp_diag_cta16.cuh"
 
 namespace mpk {
 
@@ -321,7 +322,7 @@ Variant pick_variant(int prec, int d) {
     Variant v;
     if (prec == P16 || prec == PMIX || prec == P16C) {  // half2: a lane-cell is a pair of diagonals
         if (dp <= 16) { v.DL = dp; v.G = 1; }
-        else if (dp <= 256) { v.DL = 8; v.G = dp / 8; }
+        else if (dp <= 256) { v.DL = 8; v.G = dp / 8; if (MP_CTAH_NW && dp >= MP_CTAH_MIN_DP) v.cta = MP_CTAH_NW; }
         else { v.DL = dp / 32; v.G = 32; }
         v.W = 2;
     } else if (prec == P64) {  // FP64 with the FP32 filter (mp_diag64f): one cell per lane-cell
@@ -329,11 +330,11 @@ Variant pick_variant(int prec, int d) {
         else { v.DL = 16; v.G = dp / 16; v.W = 1; }
     } else {
         if (dp <= 8) { v.DL = dp; v.G = 1; v.W = 2; }
-        else if (dp == 16) { v.DL = 16; v.G = 1; v.W = 1; }
-        else if (dp <= 512) { v.DL = 16; v.G = dp / 16; v.W = 1; if (MP_CTA_NW && dp >= 64) v.cta = MP_CTA_NW; }
+        else if (dp == 16) { v.DL = 16; v.G = 1; v.W = 1; if (MP_CTA_NW && dp >= MP_CTA_MIN_DP) v.cta = MP_CTA_NW; }
+        else if (dp <= 512) { v.DL = 16; v.G = dp / 16; v.W = 1; if (MP_CTA_NW && dp >= MP_CTA_MIN_DP) v.cta = MP_CTA_NW; }
         else { v.DL = 32; v.G = dp / 32; v.W = 1; }
     }
-    v.NC = v.cta ? 32 * v.cta / v.G : 32 / v.G * v.W;
+    v.NC = v.cta ? 32 * v.cta / v.G * v.W : 32 / v.G * v.W;
     return v;
 }
 
@@ -396,14 +397,40 @@ static long long dispatch_cta(int op, int G, const MainParams* p, int grid, cuda
         return I::blocks_per_sm();                                                         \
     }
 #if MP_CTA_NW
+#if MP_CTA_MIN_DP < 64  // measured slower than the warp kernel at d = 16 (C2: 55.9 vs 40.6 ms)
+    MP_CCASE(1) MP_CCASE(2)
+#endif
     MP_CCASE(4) MP_CCASE(8) MP_CCASE(16) MP_CCASE(32)
 #endif
 #undef MP_CCASE
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
 }
 
+template <bool SELF, int MODE>
+static long long dispatch_ctah(int op, int G, const MainParams* p, int grid, cudaStream_t s) {
+#define MP_HCCASE(g)                                                                       \
+    if (G == g) {                                                                          \
+        using I = InstCtaH<8, g, MP_CTAH_NW, SELF, MODE>;                                  \
+        if (op == 0) return (long long)I::smem();                                          \
+        if (op == 1) return (long long)I::launch(*p, grid, s);                             \
+        if (op == 3) return 1;  /* one tile per block */                                   \
+        return I::blocks_per_sm();                                                         \
+    }
+#if MP_CTAH_NW
+    MP_HCCASE(8) MP_HCCASE(16) MP_HCCASE(32)
+#endif
+#undef MP_HCCASE
+    return op == 1 ? (long long)cudaErrorInvalidValue : 0;
+}
+
 static long long dispatch(int op, int prec, bool self, int d, const MainParams* p, int grid, cudaStream_t s) {
     const Variant v = pick_variant(prec, d);
+    if (v.cta && (prec == P16 || prec == PMIX || prec == P16C)) {
+        const int md = prec == P16 ? 0 : prec == PMIX ? 1 : 2;
+        if (md == 0) return self ? dispatch_ctah<true, 0>(op, v.G, p, grid, s) : dispatch_ctah<false, 0>(op, v.G, p, grid, s);
+        if (md == 1) return self ? dispatch_ctah<true, 1>(op, v.G, p, grid, s) : dispatch_ctah<false, 1>(op, v.G, p, grid, s);
+        return self ? dispatch_ctah<true, 2>(op, v.G, p, grid, s) : dispatch_ctah<false, 2>(op, v.G, p, grid, s);
+    }
     if (v.cta) return self ? dispatch_cta<true>(op, v.G, p, grid, s) : dispatch_cta<false>(op, v.G, p, grid, s);
     if (prec == P16) return self ? dispatch_h<true, 0>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 0>(op, v.DL, v.G, p, grid, s);
     if (prec == PMIX) return self ? dispatch_h<true, 1>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 1>(op, v.DL, v.G, p, grid, s);

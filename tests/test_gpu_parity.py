@@ -262,6 +262,40 @@ def test_half_modes_ab_and_bands(ctx, prec):
     assert torch.equal(merged, full)
 
 
+@pytest.mark.parametrize("prec", ["fp16", "mixed", "fp16c"])
+@pytest.mark.parametrize("shape", [(64, 2500, 32, 8, 61), (100, 400, 16, 4, 62), (200, 300, 16, 4, 63),
+                                   (64, 700, 32, -1, 64), (130, 300, 16, -1, 65)])
+def test_half_modes_large_d(ctx, oracle_mod, prec, shape):
+    """Large d in the half modes (block-cooperative half kernel, G = 8 / 16 / 32 lanes per
+    pair): self-join (exclusion >= 0) and AB-join (-1), several tiles and ragged tails, vs the
+    oracle within the stated bound; band partials merge bit-identically to the single band."""
+    from paper_conf_ipps_juryl022_b200 import mstamp
+    d, n, m, e, seed = shape
+    T = datagen.bounded_patterns(d, n, m, seed)
+    Tr = datagen.bounded_patterns(d, n, m, seed + 1000) if e < 0 else None
+    P, I, P2 = oracle_mod.mstamp(T, m, None if e < 0 else e, Tr=Tr)
+    Pg, Ig = ctx.compute(T, m, prec, e, Tr=Tr)
+    st = _half_stats(P, I, Pg, Ig, m)
+    print(prec, shape, st)
+    assert st["median_rel"] < (0.05 if prec == "mixed" else 0.2)
+    assert np.all(np.isfinite(Pg)) and np.all((Ig >= 0) & (Ig < n))
+    assert np.all(Pg >= 0) and np.all(Pg <= 2 * math.sqrt(m) * 1.01)
+    Td = torch.from_numpy(T).cuda()
+    Trd = None if Tr is None else torch.from_numpy(Tr).cuda()
+    ee = 0 if e < 0 else e
+    kw = mstamp.key_words(d, n, prec)
+    full = torch.empty(kw, dtype=torch.int64, device="cuda")
+    ctx.partial_device(Td, m, full, 0, 1, prec, ee, Tr=Trd)
+    parts = []
+    for r in range(3):
+        k = torch.empty(kw, dtype=torch.int64, device="cuda")
+        ctx.partial_device(Td, m, k, r, 3, prec, ee, Tr=Trd)
+        parts.append(k)
+    merged = torch.stack(parts).min(dim=0).values
+    torch.cuda.synchronize()
+    assert torch.equal(merged, full)
+
+
 @pytest.mark.parametrize("prec", ["fp32", "mixed"])
 def test_c3_sampled_rows(ctx, oracle_mod, prec):
     """BASELINE config C3 at full size (self-join d=64, n=262144, m=256: the sort/scan-dominated
