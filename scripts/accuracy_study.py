@@ -68,6 +68,30 @@ def main():
             r.update(metrics(P, I, P64, I64, datagen.motif_positions(8192, 64), 16, 64))
             rows.append(r)
         c.close()
+    # BASELINE configs at full size: C2 and C3 full grids, and the C5 precision sweep on one
+    # band of a 1024-way split (the per-GPU unit of an 8-GPU run is 128 such bands) holding the
+    # planted motif, each mode against the GPU FP64 result of the same job
+    if os.environ.get("MP_ACC_FULL", "1") == "1":
+        for name in ("C2", "C3"):
+            cfg = datagen.make(name)
+            T, m, e, d, n = cfg["T"], cfg["m"], cfg["exclusion"], cfg["d"], cfg["n"]
+            P64, I64 = ctx.compute(T, m, "fp64", e)
+            for mode in MODES:
+                P, I = ctx.compute(T, m, mode, e)
+                r = dict(family=name, d=d, n=n, m=m, mode=mode, H="default")
+                r.update(metrics(P, I, P64, I64, datagen.motif_positions(n, m), d, m))
+                rows.append(r)
+        # C5's shape (d=256, m=512, exclusion 128, seed 105) on a full grid of n = 32768
+        # subsequences: every mode runs the same job as FP64 (a band of the full-size C5 would
+        # differ per mode, the tile width of the plan depends on the kernel variant)
+        d, n, m, e = 256, 32768, 512, 128
+        T = datagen.random_walk(d, n, m, 105)
+        P64, I64 = ctx.compute(T, m, "fp64", e)
+        for mode in MODES:
+            P, I = ctx.compute(T, m, mode, e)
+            r = dict(family="C5-shape", d=d, n=n, m=m, mode=mode, H="default")
+            r.update(metrics(P, I, P64, I64, datagen.motif_positions(n, m), d, m))
+            rows.append(r)
     ctx.close()
     os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
     with open(os.path.join(ROOT, "profiles", "r1_accuracy.json"), "w") as f:
@@ -76,7 +100,7 @@ def main():
     for r in rows:
         rm = "-" if r["Rm"] is None else f"{r['Rm']:.2f}"
         print(f"{r['family']:9s} {r['d']:3d} {r['n']:5d} {r['m']:4d} {r['mode']:6s} {str(r['H']):>7s} "
-              f"{r['A']:8.5f} {r['R']:7.4f} {rm:>5s}")
+              f"{r['A'] if r['A'] is None else round(r['A'], 5)!s:>8s} {r['R'] if r['R'] is None else round(r['R'], 4)!s:>7s} {rm:>5s}")
 
 
 if __name__ == "__main__":
