@@ -3,6 +3,6 @@
 #include "mp_diag_cta16.cuh"
 namespace mpk {
 #if MP_CTAH_NW
-template struct InstCtaH<8, 16, MP_CTAH_NW, false, 2>;
+template struct InstCtaH<8, 16, CtaShapeH<16>::NW, false, 2>;
 #endif
 }  // namespace mpk

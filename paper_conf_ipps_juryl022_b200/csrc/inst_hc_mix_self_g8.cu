@@ -3,6 +3,6 @@
 #include "mp_diag_cta16.cuh"
 namespace mpk {
 #if MP_CTAH_NW
-template struct InstCtaH<8, 8, MP_CTAH_NW, true, 1>;
+template struct InstCtaH<8, 8, CtaShapeH<8>::NW, true, 1>;
 #endif
 }  // namespace mpk

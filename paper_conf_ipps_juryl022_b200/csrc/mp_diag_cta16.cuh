@@ -27,26 +27,30 @@
 #include "mp_diag16.cuh"
 
 #ifndef MP_CTAH_NW
-#define MP_CTAH_NW 4       // warps per block of the block-cooperative half kernel (0: off)
+#define MP_CTAH_NW 4       // 0 switches the block-cooperative half kernel off
 #endif
 #ifndef MP_CTAH_MIN_DP
 #define MP_CTAH_MIN_DP 64  // smallest padded d that takes it
 #endif
-#ifndef MP_CTAH_SB
-#define MP_CTAH_SB 1       // steps per staging batch (one block barrier per batch)
-#endif
-#ifndef MP_CTAH_MINB
-#define MP_CTAH_MINB 4     // resident blocks per SM the register budget is sized for
-#endif
 
 namespace mpk {
+
+// Per lane-group-size launch shape (measured on one B200, Mixed, n*d^... self-joins of
+// d = 64 / 128 / 256): warps per block and steps per staging batch (one block barrier per
+// batch).  d = 64: 4 warps, SB = 2 (61.0 -> 58.9 ms); d = 128: 8 warps (45.7 -> 39.5 ms);
+// d = 256: 4 warps, SB = 1 (SB = 2: 31.3 -> 34.9 ms, 8 warps: 33.7 ms).
+template <int G> struct CtaShapeH {
+    static constexpr int NW = MP_CTAH_NW == 0 ? 0 : (G == 16 ? 8 : 4);
+    static constexpr int SB = G == 8 ? 2 : 1;
+    static constexpr int MINB = NW == 8 ? 2 : 4;   // 128 registers per thread
+};
 
 template <int DL, int G, int NW> struct CtaGeoH {
     static constexpr int NT = 32 * NW;   // threads per block
     static constexpr int NP = NT / G;    // cell pairs per block tile
     static constexpr int NCC = 2 * NP;   // cells (diagonals) per block tile
     static constexpr int D = DL * G;
-    static constexpr int SB = MP_CTAH_SB;
+    static constexpr int SB = CtaShapeH<G>::SB;
     // row slots: current batch + prefetch (+1 batch margin); column pair slots (by first
     // column): the live span [s0 - 1, s0 + SB + NCC - 2], the fixup target s0 + SB + NCC - 1
     // and the prefetch [s0 + SB + NCC, s0 + 2 SB + NCC) never share a slot
@@ -60,7 +64,7 @@ template <int DL, int G, int NW> struct CtaGeoH {
 };
 
 template <int DL, int G, int NW, bool SELF, int MODE>
-__global__ void __launch_bounds__(32 * NW, MP_CTAH_MINB)
+__global__ void __launch_bounds__(32 * NW, CtaShapeH<G>::MINB)
 mp_diag_cta_h(const MainParams p) {
     using Cg = CtaGeoH<DL, G, NW>;
     using K = unsigned long long;

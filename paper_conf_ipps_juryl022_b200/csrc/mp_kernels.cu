@@ -322,7 +322,7 @@ Variant pick_variant(int prec, int d) {
     Variant v;
     if (prec == P16 || prec == PMIX || prec == P16C) {  // half2: a lane-cell is a pair of diagonals
         if (dp <= 16) { v.DL = dp; v.G = 1; }
-        else if (dp <= 256) { v.DL = 8; v.G = dp / 8; if (MP_CTAH_NW && dp >= MP_CTAH_MIN_DP) v.cta = MP_CTAH_NW; }
+        else if (dp <= 256) { v.DL = 8; v.G = dp / 8; if (MP_CTAH_NW && dp >= MP_CTAH_MIN_DP) v.cta = v.G == 16 ? CtaShapeH<16>::NW : v.G == 8 ? CtaShapeH<8>::NW : CtaShapeH<32>::NW; }
         else { v.DL = dp / 32; v.G = 32; }
         v.W = 2;
     } else if (prec == P64) {  // FP64 with the FP32 filter (mp_diag64f): one cell per lane-cell
@@ -410,7 +410,7 @@ template <bool SELF, int MODE>
 static long long dispatch_ctah(int op, int G, const MainParams* p, int grid, cudaStream_t s) {
 #define MP_HCCASE(g)                                                                       \
     if (G == g) {                                                                          \
-        using I = InstCtaH<8, g, MP_CTAH_NW, SELF, MODE>;                                  \
+        using I = InstCtaH<8, g, CtaShapeH<g>::NW, SELF, MODE>;                                  \
         if (op == 0) return (long long)I::smem();                                          \
         if (op == 1) return (long long)I::launch(*p, grid, s);                             \
         if (op == 3) return 1;  /* one tile per block */                                   \
