@@ -1,0 +1,8 @@
+// Explicit instantiations of the block-cooperative large-d FP64 kernel (parallel build, see build.py).
+#define MP_DIAG_IMPL
+#include "mp_diag_cta64.cuh"
+namespace mpk {
+#if MP_CTA64_ON
+template struct InstCta64<16, 4, CtaShape64<4>::NW, true>;
+#endif
+}  // namespace mpk

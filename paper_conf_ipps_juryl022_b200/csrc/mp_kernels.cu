@@ -5,6 +5,7 @@
 #include "mp_diag64f.cuh"
 #include "mp_diag_cta.cuh"
 #include "mp_diag_cta16.cuh"
+#include "mp_diag_cta64.cuh"
 
 namespace mpk {
 
@@ -327,7 +328,11 @@ Variant pick_variant(int prec, int d) {
         v.W = 2;
     } else if (prec == P64) {  // FP64 with the FP32 filter (mp_diag64f): one cell per lane-cell
         if (dp <= 16) { v.DL = dp; v.G = 1; v.W = 1; }
-        else { v.DL = 16; v.G = dp / 16; v.W = 1; }
+        else {
+            v.DL = 16; v.G = dp / 16; v.W = 1;
+            if (MP_CTA64_ON && dp >= MP_CTA64_MIN_DP)
+                v.cta = v.G == 4 ? CtaShape64<4>::NW : v.G == 8 ? CtaShape64<8>::NW : v.G == 16 ? CtaShape64<16>::NW : CtaShape64<32>::NW;
+        }
     } else {
         if (dp <= 8) { v.DL = dp; v.G = 1; v.W = 2; }
         else if (dp == 16) { v.DL = 16; v.G = 1; v.W = 1; if (MP_CTA_NW && dp >= MP_CTA_MIN_DP) v.cta = MP_CTA_NW; }
@@ -423,6 +428,23 @@ static long long dispatch_ctah(int op, int G, const MainParams* p, int grid, cud
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
 }
 
+template <bool SELF>
+static long long dispatch_cta64(int op, int G, const MainParams* p, int grid, cudaStream_t s) {
+#define MP_DCCASE(g)                                                                       \
+    if (G == g) {                                                                          \
+        using I = InstCta64<16, g, CtaShape64<g>::NW, SELF>;                               \
+        if (op == 0) return (long long)I::smem();                                          \
+        if (op == 1) return (long long)I::launch(*p, grid, s);                             \
+        if (op == 3) return 1;  /* one tile per block */                                   \
+        return I::blocks_per_sm();                                                         \
+    }
+#if MP_CTA64_ON
+    MP_DCCASE(4) MP_DCCASE(8) MP_DCCASE(16) MP_DCCASE(32)
+#endif
+#undef MP_DCCASE
+    return op == 1 ? (long long)cudaErrorInvalidValue : 0;
+}
+
 static long long dispatch(int op, int prec, bool self, int d, const MainParams* p, int grid, cudaStream_t s) {
     const Variant v = pick_variant(prec, d);
     if (v.cta && (prec == P16 || prec == PMIX || prec == P16C)) {
@@ -431,6 +453,7 @@ static long long dispatch(int op, int prec, bool self, int d, const MainParams* 
         if (md == 1) return self ? dispatch_ctah<true, 1>(op, v.G, p, grid, s) : dispatch_ctah<false, 1>(op, v.G, p, grid, s);
         return self ? dispatch_ctah<true, 2>(op, v.G, p, grid, s) : dispatch_ctah<false, 2>(op, v.G, p, grid, s);
     }
+    if (v.cta && prec == P64) return self ? dispatch_cta64<true>(op, v.G, p, grid, s) : dispatch_cta64<false>(op, v.G, p, grid, s);
     if (v.cta) return self ? dispatch_cta<true>(op, v.G, p, grid, s) : dispatch_cta<false>(op, v.G, p, grid, s);
     if (prec == P16) return self ? dispatch_h<true, 0>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 0>(op, v.DL, v.G, p, grid, s);
     if (prec == PMIX) return self ? dispatch_h<true, 1>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 1>(op, v.DL, v.G, p, grid, s);
