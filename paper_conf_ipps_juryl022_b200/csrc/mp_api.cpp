@@ -225,8 +225,39 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     if (pl.nb > 0) {
         std::vector<int64_t> bb = band_blocks(pl, world);
         const long long t_begin = pl.seg[bb[rank]], t_end = pl.seg[bb[rank + 1]];
-        MP_CUDA(ctx, ensure(ctx->seg, (pl.nb + 1) * sizeof(long long)));
-        MP_CUDA(ctx, cudaMemcpyAsync(ctx->seg.p, pl.seg.data(), (pl.nb + 1) * sizeof(long long),
+        // segment-major tile order over the band's blocks [B0, B1): for row segment q the
+        // blocks with a tile in it are contiguous, [first b with qlo_b <= q, first b with
+        // qhi_b <= q), because a block's first and last rows never increase with b
+        const int64_t B0 = bb[rank], B1 = bb[rank + 1], HT = pl.H;
+        const int64_t nq = std::max<int64_t>(1, (n + HT - 1) / HT);
+        auto qlo = [&](int64_t b) {
+            const int64_t d1 = std::min(pl.dlo + b * pl.nc + pl.nc - 1, pl.dhi);
+            return std::max<int64_t>(0, -d1) / HT;
+        };
+        auto qhi = [&](int64_t b) {
+            const int64_t d0 = pl.dlo + b * pl.nc;
+            return (std::min<int64_t>(n, n - std::max<int64_t>(d0, 0)) + HT - 1) / HT;
+        };
+        auto first_b = [&](auto pred) {  // first b in [B0, B1) with pred(b) (monotone), else B1
+            int64_t lo = B0, hi = B1;
+            while (lo < hi) {
+                const int64_t mid = (lo + hi) / 2;
+                if (pred(mid)) hi = mid; else lo = mid + 1;
+            }
+            return lo;
+        };
+        std::vector<long long> qtab(2 * nq + 1);  // [q_prefix (nq + 1) | q_block0 (nq) | ...]
+        qtab[0] = 0;
+        for (int64_t q = 0; q < nq; ++q) {
+            const int64_t bs = first_b([&](int64_t b) { return qlo(b) <= q; });
+            const int64_t be = first_b([&](int64_t b) { return qhi(b) <= q; });
+            qtab[q + 1] = qtab[q] + std::max<int64_t>(0, be - bs);
+            qtab[nq + 1 + q] = bs;
+        }
+        if (qtab[nq] != t_end - t_begin) return fail(ctx, MP_ERR_INVALID, "internal: tile plan mismatch");
+        qtab.insert(qtab.end(), pl.seg.begin(), pl.seg.end());  // [.. | seg_prefix (nb + 1)]
+        MP_CUDA(ctx, ensure(ctx->seg, qtab.size() * sizeof(long long)));
+        MP_CUDA(ctx, cudaMemcpyAsync(ctx->seg.p, qtab.data(), qtab.size() * sizeof(long long),
                                      cudaMemcpyHostToDevice, s));
         MP_CUDA(ctx, ensure(ctx->counter, sizeof(unsigned long long)));
         MP_CUDA(ctx, cudaMemsetAsync(ctx->counter.p, 0, sizeof(unsigned long long), s));
@@ -240,7 +271,11 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
             mp.mu_q = ctx->mup_q.p;
             mp.mu_r = self ? ctx->mup_q.p : ctx->mup_r.p;
             mp.keys = ctx->keys.p;
-            mp.seg_prefix = (const long long*)ctx->seg.p;
+            mp.order = var.cta ? 0 : 1;   // decode_tile (mp_diag.cuh) says why
+            mp.q_prefix = (const long long*)ctx->seg.p;
+            mp.q_block0 = (const long long*)ctx->seg.p + nq + 1;
+            mp.nq = nq;
+            mp.seg_prefix = (const long long*)ctx->seg.p + 2 * nq + 1;
             mp.nb = pl.nb;
             mp.t_begin = t_begin;
             mp.t_count = t_end - t_begin;

@@ -42,6 +42,9 @@
 #endif
 #define MP_PRAGMA(x) _Pragma(#x)
 #define MP_UNROLL(n) MP_PRAGMA(unroll n)
+#ifndef MP_FUSE_LAST
+#define MP_FUSE_LAST 1   // fuse the final sort / merge layer into the scan (C2 FP32 40.35 -> 39.8 ms)
+#endif
 #ifndef MP_KEEP_DL
 #define MP_KEEP_DL 16
 #endif
@@ -150,10 +153,87 @@ template <class T, int N> __device__ __forceinline__ void sort_net(T (&v)[N]) {
     }
 }
 
+// All comparators of sort_net but the final layer's N/2 - 1 adjacent ones (i, i+1), i odd
+// (for a power of two N the generator emits that layer last).  The caller fuses that layer
+// into the inclusive scan: S_i = S_{i-1} + min(v_i, v_{i+1}), S_{i+1} = S_{i-1} + (v_i + v_{i+1})
+// -- the larger value is never formed, which moves N/2 - 1 min/max ops from the ALU pipe to
+// FADDs on the FMA pipe and halves the scan's dependency chain.
+template <int N> constexpr bool last_layer_adjacent() {
+    if (N < 4 || (N & (N - 1))) return false;
+    const BatcherNet<N> net{};
+    for (int t = 0; t < N / 2 - 1; ++t) {
+        const int c = batcher_count(N) - 1 - t;
+        if (net.a[c] != N - 3 - 2 * t || net.b[c] != N - 2 - 2 * t) return false;
+    }
+    return true;
+}
+template <class T, int N> __device__ __forceinline__ void sort_net_head(T (&v)[N]) {
+    static_assert(last_layer_adjacent<N>(), "final Batcher layer must be the adjacent odd pairs");
+    constexpr BatcherNet<N> net{};
+#pragma unroll
+    for (int c = 0; c < batcher_count(N) - (N / 2 - 1); ++c) cswap(v[net.a[c]], v[net.b[c]]);
+}
+// sort_net_head + the fused final layer + inclusive scan: v becomes S_0..S_{N-1}
+template <class T, int N> __device__ __forceinline__ void sort_scan_fused(T (&v)[N]) {
+    sort_net_head<T, N>(v);
+    T lo[N / 2], pr[N / 2];  // lo[h], pr[h]: min and sum of the pair (2h-1, 2h), h >= 1
+#pragma unroll
+    for (int h = 1; h < N / 2; ++h) {
+        lo[h] = PT<T>::vmin(v[2 * h - 1], v[2 * h]);
+        pr[h] = v[2 * h - 1] + v[2 * h];
+    }
+    // even prefix chain E_h = S_{2h} (two half chains joined), then the odd entries
+    T E[N / 2];
+    E[0] = v[0];
+    constexpr int HH = N / 4;  // second chain starts at h = HH
+#pragma unroll
+    for (int h = 1; h < HH; ++h) E[h] = E[h - 1] + pr[h];
+    T F = pr[HH];
+#pragma unroll
+    for (int h = HH + 1; h < N / 2; ++h) { E[h] = F + pr[h]; F = E[h]; }
+#pragma unroll
+    for (int h = HH; h < N / 2; ++h) E[h] = (h == HH ? pr[h] : E[h]) + E[HH - 1];
+    const T last = v[N - 1];
+#pragma unroll
+    for (int h = 1; h < N / 2; ++h) v[2 * h - 1] = E[h - 1] + lo[h];
+#pragma unroll
+    for (int h = 0; h < N / 2; ++h) v[2 * h] = E[h];
+    v[N - 1] = E[N / 2 - 1] + last;
+}
+
+// In-lane inclusive scan fused with a final layer of adjacent pairs (2h, 2h+1) left out by
+// lane_merge<..., true>: S_{2h} = E_{h-1} + min, S_{2h+1} = E_{h-1} + (v_{2h} + v_{2h+1}).
+template <class T, int DL> __device__ __forceinline__ void pair_scan(T (&v)[DL]) {
+    static_assert(DL >= 4 && (DL & (DL - 1)) == 0, "pair_scan needs a power-of-two DL >= 4");
+    constexpr int NH = DL / 2, HH = NH / 2;
+    T lo[NH], E[NH];
+#pragma unroll
+    for (int h = 0; h < NH; ++h) {
+        lo[h] = PT<T>::vmin(v[2 * h], v[2 * h + 1]);
+        E[h] = v[2 * h] + v[2 * h + 1];
+    }
+    // prefix over the pair sums in two half chains joined at the end
+#pragma unroll
+    for (int h = 1; h < HH; ++h) E[h] = E[h] + E[h - 1];
+#pragma unroll
+    for (int h = HH + 1; h < NH; ++h) E[h] = E[h] + E[h - 1];
+#pragma unroll
+    for (int h = HH; h < NH; ++h) E[h] = E[h] + E[HH - 1];
+    v[0] = lo[0];
+    v[1] = E[0];
+#pragma unroll
+    for (int h = 1; h < NH; ++h) {
+        v[2 * h] = E[h - 1] + lo[h];
+        v[2 * h + 1] = E[h];
+    }
+}
+
 // Bitonic merge of the sorted DL-blocks held by G consecutive lanes (lane-blocked order:
 // lane g ends up with ranks [g*DL, (g+1)*DL)).  The paper's group-cooperative bitonic
 // sort expressed with warp shuffles instead of shared memory.
-template <class T, int DL, int G> __device__ __forceinline__ void lane_merge(T (&v)[DL], int g) {
+// SKIP_LAST: leave out the final in-lane stage (adjacent pairs (2h, 2h+1)) for pair_scan
+template <class T, int DL, int G, bool SKIP_LAST = false>
+__device__ __forceinline__ void lane_merge(T (&v)[DL], int g) {
 #pragma unroll
     for (int p = 1; p < G; p <<= 1) {
         const bool lower = (g & p) == 0;
@@ -181,7 +261,7 @@ template <class T, int DL, int G> __device__ __forceinline__ void lane_merge(T (
         }
         // half-cleaners inside the lane
 #pragma unroll
-        for (int dist = DL / 2; dist >= 1; dist >>= 1) {
+        for (int dist = DL / 2; dist >= ((SKIP_LAST && 2 * p == G) ? 2 : 1); dist >>= 1) {
 #pragma unroll
             for (int kk = 0; kk < DL; ++kk)
                 if ((kk & dist) == 0) cswap(v[kk], v[kk + dist]);
@@ -261,6 +341,35 @@ __device__ __forceinline__ void load_dims(const T* __restrict__ rowp, int g, T (
 #pragma unroll
         for (int kk = 0; kk < DL; ++kk) out[kk] = __ldg(rowp + kk * G + g);
     }
+}
+
+// ------------------------------------------------------------------ tile order
+// Tile t of the launch -> (diagonal block b, row segment q) in the launch's order
+// (MainParams::order).  Segment-major: the tiles in flight share their rows and most columns
+// (L2 reuse of the staged statistics, faster threshold convergence: C2 FP64 106 -> 91 ms).
+// Block-major: the block-cooperative kernels' tiles in flight cover different rows, which
+// keeps their lane-local write-through merges off the same keys (segment-major measured
+// 1.1-3x slower there: C4 FP64 band 4.3 -> 12.8 s).
+__device__ __forceinline__ void decode_tile(const MainParams& p, long long t, int NC, long long& b, long long& q) {
+    if (p.order == 1) {
+        long long lo = 0, hi = p.nq;
+        while (hi - lo > 1) {
+            const long long mid = (lo + hi) >> 1;
+            if (__ldg(&p.q_prefix[mid]) <= t) lo = mid; else hi = mid;
+        }
+        q = lo;
+        b = __ldg(&p.q_block0[lo]) + (t - __ldg(&p.q_prefix[lo]));
+        return;
+    }
+    t += p.t_begin;
+    long long lo = 0, hi = p.nb;
+    while (hi - lo > 1) {
+        const long long mid = (lo + hi) >> 1;
+        if (__ldg(&p.seg_prefix[mid]) <= t) lo = mid; else hi = mid;
+    }
+    b = lo;
+    const long long delta1 = min(p.delta_lo + b * NC + NC - 1, p.delta_hi);
+    q = max(0ll, -delta1) / p.HT + (t - __ldg(&p.seg_prefix[lo]));
 }
 
 // ------------------------------------------------------------------ tile geometry
@@ -459,18 +568,11 @@ mp_diag(const MainParams p) {
         if (lane == 0) t = (long long)atomicAdd(p.counter, 1ull);
         t = __shfl_sync(FULL, t, 0);
         if (t >= p.t_count) break;
-        t += p.t_begin;
-        // block b: seg_prefix[b] <= t < seg_prefix[b+1]
-        long long lo_b = 0, hi_b = p.nb;
-        while (hi_b - lo_b > 1) {
-            const long long mid = (lo_b + hi_b) >> 1;
-            if (__ldg(&p.seg_prefix[mid]) <= t) lo_b = mid; else hi_b = mid;
-        }
-        const long long b = lo_b;
+        long long b, q;
+        decode_tile(p, t, Gm::NC, b, q);
         const long long delta0 = p.delta_lo + b * Gm::NC;
         const long long delta1 = min(delta0 + Gm::NC - 1, p.delta_hi);
         const long long rlo = max(0ll, -delta1), rhi = min(n, n - max(delta0, 0ll));
-        const long long q = rlo / HT + (t - __ldg(&p.seg_prefix[b]));
         const long long r0 = max(q * HT, rlo), r1 = min((q + 1) * HT, rhi);
 
         // the lane's W cells: diagonals and valid row ranges inside the tile
@@ -599,6 +701,9 @@ mp_diag(const MainParams p) {
             }
 #pragma unroll
             for (int u = 0; u < W; ++u) {
+                if constexpr (G == 1 && MP_FUSE_LAST && DL >= 8 && last_layer_adjacent<DL>()) {
+                    sort_scan_fused<T, DL>(S[u]);                                     // Eq. (2) sort + scan
+                } else {
                 sort_net<T, DL>(S[u]);                                               // Eq. (2) sort
                 if (G > 1) lane_merge<T, DL, G>(S[u], g);
                 // Eq. (2) inclusive scan, two independent half chains joined at the end
@@ -613,6 +718,7 @@ mp_diag(const MainParams p) {
                 } else {
 #pragma unroll
                     for (int kk = 1; kk < DL; ++kk) S[u][kk] += S[u][kk - 1];
+                }
                 }
                 if (G > 1) {
                     T tot = S[u][DL - 1];

@@ -272,17 +272,11 @@ mp_diag_h(const MainParams p) {
         if (lane == 0) t = (long long)atomicAdd(p.counter, 1ull);
         t = __shfl_sync(FULL, t, 0);
         if (t >= p.t_count) break;
-        t += p.t_begin;
-        long long lo_b = 0, hi_b = p.nb;
-        while (hi_b - lo_b > 1) {
-            const long long mid = (lo_b + hi_b) >> 1;
-            if (__ldg(&p.seg_prefix[mid]) <= t) lo_b = mid; else hi_b = mid;
-        }
-        const long long b = lo_b;
+        long long b, q;
+        decode_tile(p, t, Gm::NC, b, q);
         const long long delta0 = p.delta_lo + b * Gm::NC;
         const long long delta1 = min(delta0 + Gm::NC - 1, p.delta_hi);
         const long long rlo = max(0ll, -delta1), rhi = min(n, n - max(delta0, 0ll));
-        const long long q = rlo / HT + (t - __ldg(&p.seg_prefix[b]));
         const long long r0 = max(q * HT, rlo), r1 = min((q + 1) * HT, rhi);
 
         long long delta[2], lo[2], hi[2];

@@ -22,7 +22,7 @@
 #include "mp_diag.cuh"
 
 #ifndef MP_CTA_SB
-#define MP_CTA_SB 1   // steps per staging batch (one block barrier per batch)
+#define MP_CTA_SB 0   // steps per staging batch (one block barrier per batch); 0: per G below
 #endif
 #ifndef MP_CTA_MIN_DP
 #define MP_CTA_MIN_DP 64   // smallest padded d that takes the block-cooperative kernel
@@ -37,7 +37,8 @@ template <int DL, int G, int NW> struct CtaGeo {
     static constexpr int NT = 32 * NW;             // threads per block
     static constexpr int NCC = NT / G;             // cells (diagonals) per block tile
     static constexpr int D = DL * G;
-    static constexpr int SB = MP_CTA_SB;           // steps per staging batch
+    // steps per staging batch (measured, d = 64 / 256: SB = 2 98 / 70 ms, SB = 1 102 / 54 ms)
+    static constexpr int SB = MP_CTA_SB > 0 ? MP_CTA_SB : (G == 4 ? 2 : 1);
     // ring slots: positions of the current batch, the prefetched next one and the batch being
     // evicted stay distinct, so eviction reads and prefetch writes never touch the same slot
     static constexpr int RR = 3 * SB;
@@ -150,17 +151,11 @@ mp_diag_cta(const MainParams p) {
         __syncthreads();
         long long t = *tile_sh;
         if (t >= p.t_count) break;
-        t += p.t_begin;
-        long long lo_b = 0, hi_b = p.nb;
-        while (hi_b - lo_b > 1) {
-            const long long mid = (lo_b + hi_b) >> 1;
-            if (__ldg(&p.seg_prefix[mid]) <= t) lo_b = mid; else hi_b = mid;
-        }
-        const long long b = lo_b;
+        long long b, q;
+        decode_tile(p, t, NCC, b, q);
         const long long delta0 = p.delta_lo + b * NCC;
         const long long delta1 = min(delta0 + NCC - 1, p.delta_hi);
         const long long rlo = max(0ll, -delta1), rhi = min(n, n - max(delta0, 0ll));
-        const long long q = rlo / HT + (t - __ldg(&p.seg_prefix[b]));
         const long long r0 = max(q * HT, rlo), r1 = min((q + 1) * HT, rhi);
 
         // this thread's cell: diagonal delta, valid rows [lo, hi)
@@ -255,9 +250,14 @@ mp_diag_cta(const MainParams p) {
                     S[kk] = PT<float>::sqrt_abs(fmaf(-QT[kk], R.z * C.z, two_m));      // Eq. (1)
                 }
                 sort_net<float, DL>(S);                                               // Eq. (2)
-                lane_merge<float, DL, G>(S, g);
+                if constexpr (MP_FUSE_LAST && G > 1) {
+                    lane_merge<float, DL, G, true>(S, g);
+                    pair_scan<float, DL>(S);                                          // Eq. (2) scan
+                } else {
+                    lane_merge<float, DL, G>(S, g);
 #pragma unroll
-                for (int kk = 1; kk < DL; ++kk) S[kk] += S[kk - 1];                    // Eq. (2) scan
+                    for (int kk = 1; kk < DL; ++kk) S[kk] += S[kk - 1];                // Eq. (2) scan
+                }
                 {
                     float tot = S[DL - 1];
 #pragma unroll

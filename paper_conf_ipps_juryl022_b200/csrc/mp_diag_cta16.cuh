@@ -164,17 +164,11 @@ mp_diag_cta_h(const MainParams p) {
         __syncthreads();
         long long t = *tile_sh;
         if (t >= p.t_count) break;
-        t += p.t_begin;
-        long long lo_b = 0, hi_b = p.nb;
-        while (hi_b - lo_b > 1) {
-            const long long mid = (lo_b + hi_b) >> 1;
-            if (__ldg(&p.seg_prefix[mid]) <= t) lo_b = mid; else hi_b = mid;
-        }
-        const long long b = lo_b;
+        long long b, q;
+        decode_tile(p, t, NCC, b, q);
         const long long delta0 = p.delta_lo + b * NCC;
         const long long delta1 = min(delta0 + NCC - 1, p.delta_hi);
         const long long rlo = max(0ll, -delta1), rhi = min(n, n - max(delta0, 0ll));
-        const long long q = rlo / HT + (t - __ldg(&p.seg_prefix[b]));
         const long long r0 = max(q * HT, rlo), r1 = min((q + 1) * HT, rhi);
 
         // this thread's pair: diagonals dP, dP + 1 and their valid rows [lo_u, hi_u)
@@ -262,6 +256,10 @@ mp_diag_cta_h(const MainParams p) {
                     }
                 }
                 sort_net<__half2, DL>(S);                                                // Eq. (2)
+                if constexpr (MP_FUSE_LAST) {
+                    lane_merge<__half2, DL, G, true>(S, g);
+                    pair_scan<__half2, DL>(S);                                          // Eq. (2) scan
+                } else {
                 lane_merge<__half2, DL, G>(S, g);
                 if constexpr (DL >= 8) {  // Eq. (2) inclusive scan, two half chains joined
 #pragma unroll
@@ -273,6 +271,7 @@ mp_diag_cta_h(const MainParams p) {
                 } else {
 #pragma unroll
                     for (int kk = 1; kk < DL; ++kk) S[kk] = __hadd2(S[kk], S[kk - 1]);
+                }
                 }
                 {
                     __half2 tot = S[DL - 1];

@@ -33,9 +33,14 @@
 namespace mpk {
 
 // launch shape per lane-group size: warps per block, steps per staging batch
+#ifndef MP_CTA64_SB
+#define MP_CTA64_SB 0   // 0: per G below
+#endif
+// measured (n = 32768 / 8192 self-joins): d = 256 SB = 2 148 ms vs SB = 1 154 ms; d = 64 equal;
+// d = 512 keeps SB = 1 (the rings fill the SM)
 template <int G> struct CtaShape64 {
     static constexpr int NW = G >= 16 ? 8 : 4;
-    static constexpr int SB = 1;
+    static constexpr int SB = MP_CTA64_SB > 0 && G <= 16 ? MP_CTA64_SB : (G == 16 ? 2 : 1);
 };
 
 template <int DL, int G, int NW> struct CtaGeo64 {
@@ -125,17 +130,11 @@ mp_diag_cta64(const MainParams p) {
         __syncthreads();
         long long t = *tile_sh;
         if (t >= p.t_count) break;
-        t += p.t_begin;
-        long long lo_b = 0, hi_b = p.nb;
-        while (hi_b - lo_b > 1) {
-            const long long mid = (lo_b + hi_b) >> 1;
-            if (__ldg(&p.seg_prefix[mid]) <= t) lo_b = mid; else hi_b = mid;
-        }
-        const long long b = lo_b;
+        long long b, q;
+        decode_tile(p, t, NCC, b, q);
         const long long delta0 = p.delta_lo + b * NCC;
         const long long delta1 = min(delta0 + NCC - 1, p.delta_hi);
         const long long rlo = max(0ll, -delta1), rhi = min(n, n - max(delta0, 0ll));
-        const long long q = rlo / HT + (t - __ldg(&p.seg_prefix[b]));
         const long long r0 = max(q * HT, rlo), r1 = min((q + 1) * HT, rhi);
 
         const long long delta = delta0 + c;

@@ -15,9 +15,18 @@ struct MainParams {
     const void* mu_q;   // working-precision window means, position-major padded [pos][Dp]
     const void* mu_r;
     void* keys;         // merge keys [pos][rank] of the QUERY profile (self-join: the one profile)
-    const long long* seg_prefix;  // exclusive prefix of #segments per diagonal block (NB+1)
-    long long nb;                 // number of diagonal blocks
-    long long t_begin, t_count;   // tile range of this launch
+    // tile order.  order == 1, segment-major (warp-tile kernels): all of the band's diagonal
+    // blocks of row segment q, then q + 1, ...; tile t (0 <= t < t_count) is block
+    // q_block0[q] + (t - q_prefix[q]) of segment q, q_prefix[q] <= t < q_prefix[q + 1].
+    // order == 0, block-major (block-cooperative kernels): tile t_begin + t lies in block b
+    // with seg_prefix[b] <= t_begin + t < seg_prefix[b + 1], segment rlo_b / HT + (that - seg_prefix[b]).
+    int order;
+    const long long* q_prefix;    // exclusive prefix of #tiles per row segment (nq + 1)
+    const long long* q_block0;    // first diagonal block of the band in segment q (nq)
+    long long nq;                 // number of row segments (ceil(n / HT))
+    const long long* seg_prefix;  // exclusive prefix of #segments per diagonal block (nb + 1)
+    long long nb, t_begin;
+    long long t_count;            // tiles of this launch (the rank's band)
     unsigned long long* counter;  // zeroed before launch
     long long n;                  // subsequences
     int d, m, H;                  // dims, window, re-seed interval H (rows)
