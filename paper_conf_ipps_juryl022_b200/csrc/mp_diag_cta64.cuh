@@ -38,8 +38,11 @@ namespace mpk {
 #endif
 // measured (n = 32768 / 8192 self-joins): d = 256 SB = 2 148 ms vs SB = 1 154 ms; d = 64 equal;
 // d = 512 keeps SB = 1 (the rings fill the SM)
+#ifndef MP_CTA64_NW_SMALLG
+#define MP_CTA64_NW_SMALLG 4   // warps per block for d <= 128
+#endif
 template <int G> struct CtaShape64 {
-    static constexpr int NW = G >= 16 ? 8 : 4;
+    static constexpr int NW = G >= 16 ? 8 : MP_CTA64_NW_SMALLG;
     static constexpr int SB = MP_CTA64_SB > 0 && G <= 16 ? MP_CTA64_SB : (G == 16 ? 2 : 1);
 };
 
