@@ -45,6 +45,9 @@
 #ifndef MP_FUSE_LAST
 #define MP_FUSE_LAST 1   // fuse the final sort / merge layer into the scan (C2 FP32 40.35 -> 39.8 ms)
 #endif
+#ifndef MP_SLOW_UNROLL
+#define MP_SLOW_UNROLL 0   // 1: slow path over register-resident S, unrolled over the ranks (spills: C2 FP32 39.6 -> 48.9 ms)
+#endif
 #ifndef MP_KEEP_DL
 #define MP_KEEP_DL 16
 #endif
@@ -756,37 +759,9 @@ mp_diag(const MainParams p) {
             if (__any_sync(FULL, hit)) {
                 // Eq. (3) with the lowest-index tie rule: group min by shuffles, one leader
                 // per row / column group compares (value, index) with the ring's best.
-#pragma unroll
-                for (int u = 0; u < W; ++u)
-#pragma unroll
-                    for (int kk = 0; kk < DL; ++kk) ssc[(u * DL + kk) * 32 + lane] = active[u] ? S[u][kk] : INF;
-                __syncwarp();
-                // ranks some lane can improve (compared with the current ring bests, from
-                // shared memory so no register stays live across the slow path): one warp OR,
-                // then the loop visits only those ranks -- a slow step touches 1-2 of DL ranks
-                unsigned rk_bits = 0;
-#pragma unroll
-                for (int kk = 0; kk < DL; ++kk) {
-                    const int pl = kk * G + g;
-                    const T tr_k = rowv[pl * PSR + sr].w;
-                    bool hk = false;
-#pragma unroll
-                    for (int u = 0; u < W; ++u) {
-                        const T v = ssc[(u * DL + kk) * 32 + lane];
-                        hk |= v <= tr_k;
-                        if (SELF) hk |= v <= colv[pl * PSC + Gm::scol(col[u])].w;
-                    }
-                    rk_bits |= (unsigned)hk << kk;
-                }
-                rk_bits = __reduce_or_sync(FULL, rk_bits);
                 DMask mark_r = 0, mark_c = 0;  // ring slots this lane's leader updates dirtied
-#pragma unroll 1
-                for (; rk_bits != 0; rk_bits &= rk_bits - 1) {
-                    const int kk = __ffs(rk_bits) - 1;
+                auto rank_update = [&](const int kk, const T (&v)[W]) {
                     const int pl = kk * G + g;
-                    T v[W];
-#pragma unroll
-                    for (int u = 0; u < W; ++u) v[u] = ssc[(u * DL + kk) * 32 + lane];
                     // skip ranks (and sides) no lane can improve: most slow steps touch 1-2 ranks
                     T vmin_l = v[0];
 #pragma unroll
@@ -798,7 +773,7 @@ mp_diag(const MainParams p) {
                         for (int u = 0; u < W; ++u) need_c |= v[u] <= colv[pl * PSC + Gm::scol(col[u])].w;
                         need_c = __any_sync(FULL, need_c);
                     }
-                    if (!need_r && !need_c) continue;
+                    if (!need_r && !need_c) return;
                     // row group: W cells per lane x CA lanes
                     T vr = v[0];
 #pragma unroll
@@ -846,6 +821,65 @@ mp_diag(const MainParams p) {
                             }
                         }
                     }
+                };
+                if constexpr (MP_SLOW_UNROLL) {
+                    // ranks some lane can improve, from registers (S stays live; the ring's
+                    // current bests are re-read); then a fully unrolled pass over the ranks
+                    // with a warp-uniform skip: no shared-memory round trip of S
+                    unsigned rk_bits = 0;
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) {
+                        const int pl = kk * G + g;
+                        const T tr_k = rowv[pl * PSR + sr].w;
+                        bool hk = false;
+#pragma unroll
+                        for (int u = 0; u < W; ++u) {
+                            hk |= active[u] && S[u][kk] <= tr_k;
+                            if (SELF) hk |= active[u] && S[u][kk] <= colv[pl * PSC + Gm::scol(col[u])].w;
+                        }
+                        rk_bits |= (unsigned)hk << kk;
+                    }
+                    rk_bits = __reduce_or_sync(FULL, rk_bits);
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) {
+                        if (!((rk_bits >> kk) & 1u)) continue;
+                        T v[W];
+#pragma unroll
+                        for (int u = 0; u < W; ++u) v[u] = active[u] ? S[u][kk] : INF;
+                        rank_update(kk, v);
+                    }
+                } else {
+#pragma unroll
+                for (int u = 0; u < W; ++u)
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) ssc[(u * DL + kk) * 32 + lane] = active[u] ? S[u][kk] : INF;
+                __syncwarp();
+                // ranks some lane can improve (compared with the current ring bests, from
+                // shared memory so no register stays live across the slow path): one warp OR,
+                // then the loop visits only those ranks -- a slow step touches 1-2 of DL ranks
+                unsigned rk_bits = 0;
+#pragma unroll
+                for (int kk = 0; kk < DL; ++kk) {
+                    const int pl = kk * G + g;
+                    const T tr_k = rowv[pl * PSR + sr].w;
+                    bool hk = false;
+#pragma unroll
+                    for (int u = 0; u < W; ++u) {
+                        const T v = ssc[(u * DL + kk) * 32 + lane];
+                        hk |= v <= tr_k;
+                        if (SELF) hk |= v <= colv[pl * PSC + Gm::scol(col[u])].w;
+                    }
+                    rk_bits |= (unsigned)hk << kk;
+                }
+                rk_bits = __reduce_or_sync(FULL, rk_bits);
+#pragma unroll 1
+                for (; rk_bits != 0; rk_bits &= rk_bits - 1) {
+                    const int kk = __ffs(rk_bits) - 1;
+                    T v[W];
+#pragma unroll
+                    for (int u = 0; u < W; ++u) v[u] = ssc[(u * DL + kk) * 32 + lane];
+                    rank_update(kk, v);
+                }
                 }
                 dmask_r |= or_reduce(mark_r);
                 dmask_c |= or_reduce(mark_c);

@@ -122,11 +122,14 @@ def test_reseed_interval_independent(ctx, oracle_mod, prec):
 
 @pytest.mark.parametrize("prec", ["fp64", "fp32"])
 @pytest.mark.parametrize("world", [2, 3, 8])
-def test_bands_bit_identical(ctx, prec, world):
+@pytest.mark.parametrize("d", [6, 70])
+def test_bands_bit_identical(ctx, prec, world, d):
     """Band partition emulated on one GPU: per-rank partial keys merged by MIN (the NCCL
-    collective's semantics) are bit-identical to the single-band result."""
+    collective's semantics) are bit-identical to the single-band result.
+    d = 6: warp-tile kernels (segment-major tile order); d = 70: block-cooperative kernels
+    (block-major order, padded dims)."""
     from paper_conf_ipps_juryl022_b200 import mstamp
-    d, n, m = 6, 3000, 32
+    n, m = (3000, 32) if d < 32 else (1200, 16)
     T = torch.from_numpy(datagen.random_walk(d, n, m, 34)).cuda()
     cnt = d * n
     kw = mstamp.key_words(d, n, prec)
