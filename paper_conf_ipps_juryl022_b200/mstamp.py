@@ -150,8 +150,12 @@ class Context:
             raise MPError(st, f"{what}: {load().mp_last_error(self._ctx).decode()}")
 
     # ---- host memory
-    def compute(self, T, m, prec="fp32", exclusion=-1, Tr=None):
-        """P (d,n) float64 and I (d,n) int64 from host series T (d,L) [and Tr]."""
+    def compute(self, T, m, prec="fp32", exclusion=-1, Tr=None, out=None):
+        """P (d,n) float64 and I (d,n) int64 from host series T (d,L) [and Tr].
+
+        out: optional preallocated (P, I) host arrays (C-contiguous float64 / int64, shape
+        (d, n)), e.g. views of pinned buffers, so repeated calls skip the allocation and the
+        page faults of fresh output memory."""
         T = np.ascontiguousarray(T, dtype=np.float64)
         if T.ndim == 1:
             T = T[None, :]
@@ -164,8 +168,14 @@ class Context:
                 Tr_ = Tr_[None, :]
             if Tr_.shape != T.shape:
                 raise MPError(1, "AB-join needs equal shapes")
-        P = np.empty((d, n), dtype=np.float64)
-        I = np.empty((d, n), dtype=np.int64)
+        if out is None:
+            P = np.empty((d, n), dtype=np.float64)
+            I = np.empty((d, n), dtype=np.int64)
+        else:
+            P, I = out
+            if (P.shape != (d, n) or I.shape != (d, n) or P.dtype != np.float64 or I.dtype != np.int64
+                    or not P.flags.c_contiguous or not I.flags.c_contiguous):
+                raise MPError(1, "out must be C-contiguous float64 / int64 arrays of shape (d, n)")
         st = load().mp_compute(self._ctx, T.ctypes.data_as(ctypes.c_void_p),
                                None if Tr_ is None else Tr_.ctypes.data_as(ctypes.c_void_p),
                                d, n, m, _prec(prec), int(exclusion),
