@@ -3,6 +3,6 @@
 #include "mp_diag_cta64.cuh"
 namespace mpk {
 #if MP_CTA64_ON
-template struct InstCta64<16, 32, CtaShape64<32>::NW, false>;
+template struct InstCta64<MP_CTA64_DL, 32, CtaShape64<32>::NW, false>;
 #endif
 }  // namespace mpk

@@ -3,6 +3,6 @@
 #include "mp_diag_cta64.cuh"
 namespace mpk {
 #if MP_CTA64_ON
-template struct InstCta64<16, 4, CtaShape64<4>::NW, true>;
+template struct InstCta64<MP_CTA64_DL, 4, CtaShape64<4>::NW, true>;
 #endif
 }  // namespace mpk

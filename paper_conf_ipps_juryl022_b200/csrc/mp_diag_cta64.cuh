@@ -26,6 +26,9 @@
 #ifndef MP_CTA64_ON
 #define MP_CTA64_ON 1       // 0 switches the block-cooperative FP64 kernel off
 #endif
+#ifndef MP_CTA64_DL
+#define MP_CTA64_DL 16      // dims per lane (G = d_pad / DL lanes per cell)
+#endif
 #ifndef MP_CTA64_MIN_DP
 #define MP_CTA64_MIN_DP 64  // smallest padded d that takes it
 #endif

@@ -330,8 +330,11 @@ Variant pick_variant(int prec, int d) {
         if (dp <= 16) { v.DL = dp; v.G = 1; v.W = 1; }
         else {
             v.DL = 16; v.G = dp / 16; v.W = 1;
-            if (MP_CTA64_ON && dp >= MP_CTA64_MIN_DP)
+            if (MP_CTA64_ON && dp >= MP_CTA64_MIN_DP && dp / MP_CTA64_DL <= 32) {
+                v.DL = MP_CTA64_DL;
+                v.G = dp / v.DL;
                 v.cta = v.G == 4 ? CtaShape64<4>::NW : v.G == 8 ? CtaShape64<8>::NW : v.G == 16 ? CtaShape64<16>::NW : CtaShape64<32>::NW;
+            }
         }
     } else {
         if (dp <= 8) { v.DL = dp; v.G = 1; v.W = 2; }
@@ -432,7 +435,7 @@ template <bool SELF>
 static long long dispatch_cta64(int op, int G, const MainParams* p, int grid, cudaStream_t s) {
 #define MP_DCCASE(g)                                                                       \
     if (G == g) {                                                                          \
-        using I = InstCta64<16, g, CtaShape64<g>::NW, SELF>;                               \
+        using I = InstCta64<MP_CTA64_DL, g, CtaShape64<g>::NW, SELF>;                      \
         if (op == 0) return (long long)I::smem();                                          \
         if (op == 1) return (long long)I::launch(*p, grid, s);                             \
         if (op == 3) return 1;  /* one tile per block */                                   \
