@@ -28,6 +28,22 @@ template <> struct PT<__half2> {
     static __device__ __forceinline__ __half2 vmax(__half2 a, __half2 b) { return __hmax2(a, b); }
 };
 
+// D of a cell pair (Eq. 1): D^2 = 2m - QT (a_i a_j) by a mixed-precision FMA (half operands,
+// FP32 result: FHFMA, .H0/.H1 selectors, no half rounding of D^2 and no conversion before the
+// FP32 square root), then sqrt of |D^2| (reading G5) rounded to half (reading G14).
+__device__ __forceinline__ __half2 dist_pair(__half2 qt, __half2 aa, float two_m) {
+    float lo, hi;
+    asm("{\n .reg .f16 q0, q1, a0, a1;\n mov.b32 {q0, q1}, %2;\n mov.b32 {a0, a1}, %3;\n"
+        " neg.f16 q0, q0;\n neg.f16 q1, q1;\n"
+        " fma.rn.f32.f16 %0, q0, a0, %4;\n fma.rn.f32.f16 %1, q1, a1, %4;\n}"
+        : "=f"(lo), "=f"(hi)
+        : "r"(*reinterpret_cast<const unsigned*>(&qt)), "r"(*reinterpret_cast<const unsigned*>(&aa)), "f"(two_m));
+    float slo, shi;
+    asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(slo) : "f"(fabsf(lo)));
+    asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(shi) : "f"(fabsf(hi)));
+    return __floats2half2_rn(slo, shi);
+}
+
 struct alignas(8) RH { __half df, dg, a, t; };   // row ring entry (one position)
 struct alignas(16) H4 { __half2 x, y, z, w; };   // column ring entry (pair c, c+1)
 
@@ -196,7 +212,7 @@ mp_diag_h(const MainParams p) {
     const long long n = p.n;
     const int d = p.d, m = p.m, H = p.H, HT = p.HT;
     const int n32 = (int)n;
-    const __half2 two_m = __float2half2_rn((float)(2 * m));
+    const float two_mf = (float)(2 * m);
     const float FINF = __int_as_float(0x7f800000);
     const __half HZERO = __float2half(0.f), HINF = __ushort_as_half(0x7c00);
 
@@ -335,7 +351,7 @@ mp_diag_h(const MainParams p) {
                     const RH R = rowv[pl * PSR + sr];
                     const H4 C = colv[pl * PSC + scn];
                     if (upd[0]) QT[kk] = __hfma2(__half2half2(R.df), C.y, __hfma2(C.x, __half2half2(R.dg), QT[kk]));
-                    S[kk] = h2sqrt(__habs2(__hfma2(__hneg2(QT[kk]), __hmul2(__half2half2(R.a), C.z), two_m)));
+                    S[kk] = dist_pair(QT[kk], __hmul2(__half2half2(R.a), C.z), two_mf);
                     th[kk] = SELF ? __hmax2(__half2half2(R.t), C.w) : __half2half2(R.t);
                 }
             } else {  // the two cells of the pair are at different phases (tile / diagonal start)
@@ -346,7 +362,7 @@ mp_diag_h(const MainParams p) {
                     const RH R = rowv[pl * PSR + sr];
                     const H4 C = colv[pl * PSC + scn];
                     QT[kk] = __hfma2(msk, __hfma2(__half2half2(R.df), C.y, __hmul2(C.x, __half2half2(R.dg))), QT[kk]);
-                    S[kk] = h2sqrt(__habs2(__hfma2(__hneg2(QT[kk]), __hmul2(__half2half2(R.a), C.z), two_m)));
+                    S[kk] = dist_pair(QT[kk], __hmul2(__half2half2(R.a), C.z), two_mf);
                     th[kk] = SELF ? __hmax2(__half2half2(R.t), C.w) : __half2half2(R.t);
                 }
             }

@@ -90,7 +90,7 @@ mp_diag_cta_h(const MainParams p) {
     const long long n = p.n;
     const int n32 = (int)n;
     const int d = p.d, m = p.m, H = p.H, HT = p.HT;
-    const __half2 two_m = __float2half2_rn((float)(2 * m));
+    const float two_mf = (float)(2 * m);
     const float FINF = __int_as_float(0x7f800000);
     const __half HZERO = __float2half(0.f), HINF = __ushort_as_half(0x7c00);
     const int tid = threadIdx.x;
@@ -240,7 +240,7 @@ mp_diag_cta_h(const MainParams p) {
                         const RH R = rowv[sr * D + pl];
                         const H4 C = colv[sc * D + pl];
                         if (upd[0]) QT[kk] = __hfma2(__half2half2(R.df), C.y, __hfma2(C.x, __half2half2(R.dg), QT[kk]));  // Eq. (1)
-                        S[kk] = h2sqrt(__habs2(__hfma2(__hneg2(QT[kk]), __hmul2(__half2half2(R.a), C.z), two_m)));     // Eq. (1)
+                        S[kk] = dist_pair(QT[kk], __hmul2(__half2half2(R.a), C.z), two_mf);     // Eq. (1)
                         th[kk] = SELF ? __hmax2(__half2half2(R.t), C.w) : __half2half2(R.t);
                     }
                 } else {  // the two cells are at different phases (diagonal start / tile start)
@@ -251,7 +251,7 @@ mp_diag_cta_h(const MainParams p) {
                         const RH R = rowv[sr * D + pl];
                         const H4 C = colv[sc * D + pl];
                         QT[kk] = __hfma2(msk, __hfma2(__half2half2(R.df), C.y, __hmul2(C.x, __half2half2(R.dg))), QT[kk]);
-                        S[kk] = h2sqrt(__habs2(__hfma2(__hneg2(QT[kk]), __hmul2(__half2half2(R.a), C.z), two_m)));
+                        S[kk] = dist_pair(QT[kk], __hmul2(__half2half2(R.a), C.z), two_mf);
                         th[kk] = SELF ? __hmax2(__half2half2(R.t), C.w) : __half2half2(R.t);
                     }
                 }
