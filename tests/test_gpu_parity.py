@@ -201,6 +201,24 @@ def _half_stats(P_or, I_or, P, I, m):
                 max_rel=float(rel.max()), recall=float((I == I_or)[fin].mean()))
 
 
+def test_compute_out_buffers(ctx):
+    """Context.compute(out=) (preallocated, e.g. pinned, host outputs: the bench's e2e leg)
+    returns exactly what the allocating call returns; malformed outputs are rejected."""
+    from paper_conf_ipps_juryl022_b200 import mstamp
+    d, n, m = 3, 700, 16
+    T = datagen.random_walk(d, n, m, 71)
+    P0, I0 = ctx.compute(T, m, "fp32", 4)
+    outs = (torch.empty((d, n), dtype=torch.float64, pin_memory=True).numpy(),
+            torch.empty((d, n), dtype=torch.int64, pin_memory=True).numpy())
+    P1, I1 = ctx.compute(T, m, "fp32", 4, out=outs)
+    assert P1 is outs[0] and I1 is outs[1]
+    assert np.array_equal(P0, P1) and np.array_equal(I0, I1)
+    with pytest.raises(mstamp.MPError):
+        ctx.compute(T, m, "fp32", 4, out=(np.empty((d, n + 1)), np.empty((d, n), dtype=np.int64)))
+    with pytest.raises(mstamp.MPError):
+        ctx.compute(T, m, "fp32", 4, out=(np.empty((d, n)), np.empty((d, n), dtype=np.int32)))
+
+
 @pytest.mark.parametrize("prec", ["fp16", "mixed", "fp16c"])
 def test_half_modes_c1(ctx, oracle_mod, c1_oracle, prec):
     """FP16 / Mixed: no tolerance gate (parity unpinned); the
