@@ -42,6 +42,9 @@
 #endif
 #define MP_PRAGMA(x) _Pragma(#x)
 #define MP_UNROLL(n) MP_PRAGMA(unroll n)
+#ifndef MP_CA_W2
+#define MP_CA_W2 4   // lanes per row group for two cells per lane (half kernel d <= 16, FP32 d <= 8)
+#endif
 #ifndef MP_FUSE_LAST
 #define MP_FUSE_LAST 1   // fuse the final sort / merge layer into the scan (C2 FP32 40.35 -> 39.8 ms)
 #endif
@@ -382,7 +385,7 @@ constexpr int ilog2(int x) { int l = 0; while ((1 << l) < x) ++l; return l; }
 template <int G, int W> struct Geo {
     static constexpr int NL = 32 / G;                                   // lane-cells per warp
     // lane-cells per row group: 8 x 4 (rows x lanes) for one cell per lane, else 4 columns
-    static constexpr int CA = (W == 1 && NL == 32) ? 8 : NL >= 16 ? 4 : (NL >= 4 ? 2 : 1);
+    static constexpr int CA = (W == 1 && NL == 32) ? 8 : (W == 2 && NL == 32) ? MP_CA_W2 : NL >= 16 ? 4 : (NL >= 4 ? 2 : 1);
     static constexpr int RA = NL / CA;                                   // distinct rows per step
     static constexpr int CW = CA * W;                                    // distinct columns per step
     static constexpr int NC = NL * W;                                    // cells (diagonals) per warp
