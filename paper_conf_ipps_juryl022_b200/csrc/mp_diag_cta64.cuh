@@ -15,7 +15,10 @@
 // d >= 64 a warp-private ring held only 2-8 cells per warp and 3-6 warps per SM.  Here the NW
 // warps of a block step through one tile together: the block's NT/G cells are consecutive
 // diagonals in the SAME row, so per step the block stages one row and one column position
-// into rings shared by all its warps.  Profile updates write through (no eviction pass); the
+// into rings shared by all its warps.  Row updates (all cells of a step share the row) merge
+// into a shared-memory FP64 key ring (128-bit CAS) that reaches the global key once per
+// (row, rank) when the row leaves the ring (d <= 256; d = 512 writes through, the ring does
+// not fit); column updates write through to the global key.  The
 // FP32 filter thresholds in the ring are hints that only ever sit at or above the true
 // (widened) best: a racing store can only leave one higher, which costs an extra exact pass,
 // never a missed update.  Thresholds enter the ring as the key's FP64 value (cp.async into the
@@ -44,10 +47,42 @@ namespace mpk {
 #ifndef MP_CTA64_NW_SMALLG
 #define MP_CTA64_NW_SMALLG 4   // warps per block for d <= 128
 #endif
+#ifndef MP_CTA64_QN
+#define MP_CTA64_QN 256   // per-block queue of global write-through merges, flushed once per batch (0: off)
+#endif
+#ifndef MP_CTA64_ROWKEY
+#define MP_CTA64_ROWKEY 1   // row bests in a shared-memory key ring (d <= 256), merged at eviction
+#endif
 template <int G> struct CtaShape64 {
     static constexpr int NW = G >= 16 ? 8 : MP_CTA64_NW_SMALLG;
-    static constexpr int SB = MP_CTA64_SB > 0 && G <= 16 ? MP_CTA64_SB : (G == 16 ? 2 : 1);
+    // row key ring: the rows of a block tile are shared by all its cells, so their merges go
+    // to shared memory (128-bit CAS) and reach the global key once per (row, rank) per tile;
+    // it does not fit next to the d = 512 rings
+    static constexpr bool ROWKEY = MP_CTA64_ROWKEY && G <= 16;
+    static constexpr int SB = MP_CTA64_SB > 0 && G <= 16 ? MP_CTA64_SB : ((G == 16 && !ROWKEY) ? 2 : 1);
 };
+
+struct alignas(16) PendQ { unsigned long long key; double v; unsigned idx, pad0, pad1, pad2; };
+
+// lexicographic (value, index) min into a shared-memory FP64 key (128-bit CAS)
+__device__ __forceinline__ void smem_merge64(K64* p, double v, unsigned i) {
+    const unsigned long long nv = (unsigned long long)__double_as_longlong(v), ni = i;
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(p);
+    ulonglong2 old;
+    asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];" : "=l"(old.x), "=l"(old.y) : "r"(sa) : "memory");
+    while (nv < old.x || (nv == old.x && ni < old.y)) {
+        unsigned long long ox, oy;
+        asm volatile(
+            "{\n .reg .b128 c, n, o;\n mov.b128 c, {%2, %3};\n mov.b128 n, {%4, %5};\n"
+            " atom.shared.cas.b128 o, [%6], c, n;\n mov.b128 {%0, %1}, o;\n}\n"
+            : "=l"(ox), "=l"(oy)
+            : "l"(old.x), "l"(old.y), "l"(nv), "l"(ni), "r"(sa)
+            : "memory");
+        if (ox == old.x && oy == old.y) break;
+        old.x = ox;
+        old.y = oy;
+    }
+}
 
 template <int DL, int G, int NW> struct CtaGeo64 {
     static constexpr int NT = 32 * NW;   // threads per block
@@ -57,7 +92,8 @@ template <int DL, int G, int NW> struct CtaGeo64 {
     // current batch + prefetch never share a slot (write-through: no eviction to wait for)
     static constexpr int RR = 3 * SB;
     static constexpr int RC = 3 * SB + NCC - 1;
-    static constexpr size_t bytes = (size_t)(RR + RC) * D * sizeof(E64) + 16;
+    static constexpr bool ROWKEY = CtaShape64<G>::ROWKEY;
+    static constexpr size_t bytes = (size_t)(RR + RC) * D * sizeof(E64) + (ROWKEY ? (size_t)RR * D * sizeof(K64) + 16 * ((RR * 4 + 15) / 16) : 0) + (size_t)MP_CTA64_QN * sizeof(PendQ) + 32;
 };
 
 template <int DL, int G, int NW, bool SELF>
@@ -69,9 +105,15 @@ mp_diag_cta64(const MainParams p) {
     constexpr int D = Cg::D, NCC = Cg::NCC, RR = Cg::RR, RC = Cg::RC, SB = Cg::SB, NT = Cg::NT;
 
     extern __shared__ __align__(16) unsigned char smem_raw[];
+    constexpr bool ROWKEY = Cg::ROWKEY;
     E64* rowv = reinterpret_cast<E64*>(smem_raw);
     E64* colv = rowv + (size_t)RR * D;
-    long long* tile_sh = reinterpret_cast<long long*>(colv + (size_t)RC * D);
+    K64* rowk = reinterpret_cast<K64*>(colv + (size_t)RC * D);                      // ROWKEY: [RR][D]
+    unsigned* rdirty = reinterpret_cast<unsigned*>(rowk + (ROWKEY ? (size_t)RR * D : 0));
+    constexpr int QN = MP_CTA64_QN;
+    PendQ* pq = reinterpret_cast<PendQ*>(reinterpret_cast<unsigned char*>(rdirty) + (ROWKEY ? 16 * ((RR * 4 + 15) / 16) : 0));
+    long long* tile_sh = reinterpret_cast<long long*>(pq + QN);
+    unsigned* qn = reinterpret_cast<unsigned*>(tile_sh + 1);   // queued merges (monotone)
 
     const double4* __restrict__ st_q = reinterpret_cast<const double4*>(p.st_q);
     const double4* __restrict__ st_r = reinterpret_cast<const double4*>(p.st_r);
@@ -90,6 +132,22 @@ mp_diag_cta64(const MainParams p) {
     const double margin = 1.0 + ldexp(1.0, -20) + (double)d * ldexp(1.0, -22);
     const int tid = threadIdx.x;
     const int c = tid / G, g = tid & (G - 1);  // cell of the block tile, lane within the cell
+    if (tid == 0) *qn = 0u;
+    unsigned qbase = 0;                                         // block-uniform: flushed so far
+    // global write-through merge, queued when there is room (the queue is flushed by all threads
+    // at the batch end, so the L2 round trips of the CAS loops overlap instead of serialising
+    // behind the lanes that hit)
+    auto merge_q = [&](size_t key, double v, unsigned idx) {
+        if constexpr (QN > 0) {
+            const unsigned slot = atomicAdd(qn, 1u);
+            if (slot - qbase < (unsigned)QN) {
+                PendQ& e = pq[slot % QN];
+                e.key = key; e.v = v; e.idx = idx;
+                return;
+            }
+        }
+        KO::merge(keys + key, v, idx);
+    };
 
     const int off_r = ((n32 + RR) / RR) * RR, off_c = ((n32 + RC) / RC) * RC;
     auto rslot = [&](int pos) { return (pos + off_r) % RR; };
@@ -116,6 +174,28 @@ mp_diag_cta64(const MainParams p) {
             }
             if (pos >= 0 && pos < n32 && rk < d && want_thr) cp_async8(&dst->thr, &keys[(size_t)pos * d + rk].v);
             else *reinterpret_cast<double*>(&dst->thr) = -INF;  // never hit
+            if (ROWKEY && is_row) {
+                const int sl = rslot(pos);
+                if (pl == 0) rdirty[sl] = 0;
+                K64* kd = &rowk[sl * D + pl];
+                if (pos >= 0 && pos < n32 && rk < d) cp_async16(kd, &keys[(size_t)pos * d + rk]);
+                else { kd->v = EMPTY64V; kd->i = EMPTY64I; }
+            }
+        }
+    };
+    // ROWKEY: merge the dirty row keys of positions [p_lo, p_hi) into the global keys
+    auto evict_rows = [&](int base, int p_lo, int p_hi) {
+        const int cnt = p_hi - p_lo;
+        for (int e = tid; e < cnt * D; e += NT) {
+            const int pi = e / D, pl = e - pi * D;
+            const int pos = base + p_lo + pi;
+            if (pos < 0 || pos >= n32) continue;
+            const int sl = rslot(pos);
+            if (rdirty[sl] == 0) continue;
+            const int rk = rank_of_plane<DL, G>(pl);
+            if (rk >= d) continue;
+            const K64 kv = rowk[sl * D + pl];
+            if (kv.v < EMPTY64V) KO::merge(keys + (size_t)pos * d + rk, __longlong_as_double((long long)kv.v), (unsigned)kv.i);
         }
     };
     // after this thread's copies landed: FP32 filter thresholds (rounded up, widened)
@@ -204,6 +284,7 @@ mp_diag_cta64(const MainParams p) {
                 if (row > lo && row < hi) seed_cell(row);
                 seeded_step = s0;
             }
+            if (ROWKEY && s0 > 0) evict_rows(R0, s0 - SB, s0);  // the previous batch's rows
             const int nxt = min(s0 + 2 * SB, nrows);
             const int r_lo = row_in, c_lo = col_in;
             stage(true, R0, row_in, nxt);
@@ -291,13 +372,18 @@ mp_diag_cta64(const MainParams p) {
                     if (rk >= d) continue;
                     float& thr_r = rowv[sr * D + pl].thr;
                     if (v <= (double)thr_r) {
-                        KO::merge(keys + (size_t)row * d + rk, v, (unsigned)col);
+                        if constexpr (ROWKEY) {
+                            smem_merge64(&rowk[sr * D + pl], v, (unsigned)col);
+                            rdirty[sr] = 1;
+                        } else {
+                            merge_q((size_t)row * d + rk, v, (unsigned)col);
+                        }
                         thr_r = fminf(thr_r, __double2float_ru(v * margin));
                     }
                     if (SELF) {
                         float& thr_c = colv[sc * D + pl].thr;
                         if (v <= (double)thr_c) {
-                            KO::merge(keys + (size_t)col * d + rk, v, (unsigned)row);
+                            merge_q((size_t)col * d + rk, v, (unsigned)row);
                             thr_c = fminf(thr_c, __double2float_ru(v * margin));
                         }
                     }
@@ -307,7 +393,20 @@ mp_diag_cta64(const MainParams p) {
             fixup(true, R0, r_lo, row_in);     // ... so it converts the thresholds it staged
             fixup(false, C0, c_lo, col_in);
             __syncthreads();                   // publish; this batch's reads are all done
+            if constexpr (QN > 0) {            // flush the queued merges with every thread
+                const unsigned qnow = *reinterpret_cast<volatile unsigned*>(qn);
+                if (qnow != qbase) {
+                    const unsigned qend = min(qnow, qbase + (unsigned)QN);
+                    for (unsigned j = qbase + tid; j < qend; j += NT) {
+                        const PendQ e = pq[j % QN];
+                        KO::merge(keys + e.key, e.v, e.idx);
+                    }
+                    qbase = qnow;
+                    __syncthreads();           // queue slots free again
+                }
+            }
         }
+        if (ROWKEY && nrows > 0) evict_rows(R0, ((nrows - 1) / SB) * SB, row_in);  // the last rows
     }
 }
 
