@@ -305,10 +305,13 @@ def main():
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream(dev)
 
+    last = {}
+
     def one_step(prec):
         """One pass of the whole hot path; returns (device ms, main-kernel ms)."""
         P = torch.empty(d, n, dtype=torch.float64, device=dev)
         I = torch.empty(d, n, dtype=torch.int64, device=dev)
+        last["P"], last["I"], last["prec"] = P, I, prec
         flush.fill_(1)
         if world > 1:
             dist.barrier()
@@ -347,6 +350,16 @@ def main():
         return tot.item() / steps, statistics.mean(kms), clocks
 
     ms, kms, clocks = timed(args.precision, args.steps, args.warmup, sample_clocks=True)
+    merge_check = None
+    if world > 1 and rank == 0:
+        # outside the timed region: the merged N-rank result must equal the 1-GPU result bit
+        # for bit (fixed tile plan, lexicographic MINLOC merge: DESIGN.md section 10)
+        P1 = torch.empty(d, n, dtype=torch.float64, device=dev)
+        I1 = torch.empty(d, n, dtype=torch.int64, device=dev)
+        ctx.compute_device(T, m, P1, I1, args.precision, e, Tr=Tr, stream=stream)
+        torch.cuda.synchronize()
+        merge_check = {"bit_identical_to_1gpu": bool(torch.equal(P1, last["P"]) and torch.equal(I1, last["I"]))}
+        del P1, I1
     dn2 = d * n * n
     value = dn2 / (ms * 1e-3)
 
@@ -423,6 +436,8 @@ def main():
                 "e2e": e2e, "gpu_launches": launches_per_step(args.precision, self_join) * args.steps,
                 "clocks": clocks, "per_precision": per_prec, "per_config_band": per_cfg or None,
                 "computed_cells_per_s": cells * d / (ms * 1e-3)}
+        if merge_check is not None:
+            line["merge_check"] = merge_check
         print(json.dumps(line), flush=True)
     ctx.close()
     if world > 1:
