@@ -39,6 +39,22 @@ UNIT = "cells*dims/s"
 SM_COUNT = 148
 ALU_LANES = 64          # ALU-pipe lanes per SM per clock (FMNMX/FSETP/FSEL), B300_MICROARCH "alu rt=2/SMSP"
 NOMINAL_SM_MHZ = 1965.0
+PIPE_PEAKS_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "r1_pipe_peaks.json")
+
+
+def alu_lanes():
+    """ALU-pipe lanes per SM per clock: measured by scripts/pipe_peaks.cu on a B200 (FMNMX with
+    8 independent chains per thread, 2048 threads/SM), else the nominal 64."""
+    try:
+        with open(PIPE_PEAKS_PATH) as f:
+            return float(json.load(f)["fmnmx_alu"]["lanes_per_sm_clk"]), "measured"
+    except (OSError, KeyError, ValueError):
+        return float(ALU_LANES), "nominal"
+
+
+def alu_peak_ops(sm_mhz=None):
+    lanes, _ = alu_lanes()
+    return SM_COUNT * lanes * (sm_mhz or NOMINAL_SM_MHZ) * 1e6
 
 
 def batcher_ce(N: int) -> int:
@@ -157,7 +173,7 @@ def alu_ops_mode(d: int, self_join: bool, prec: str) -> float:
 _PROBE_CACHE = {}
 
 
-def band_probe(ctx, torch, dev, name: str, prec: str, target_cell_dims: float = 3e11):
+def band_probe(ctx, torch, dev, name: str, prec: str, target_cell_dims: float = 3e11, peak=None):
     """Throughput of one diagonal band of a larger BASELINE config at its full input size: the
     unit one rank computes under bench.py --gpus N (mp_partial_device), timed by the library's
     CUDA events around the main kernel.  The band is the middle one of a W-way equal-cell split
@@ -186,7 +202,7 @@ def band_probe(ctx, torch, dev, name: str, prec: str, target_cell_dims: float = 
     del keys
     cd = int(bc[r]) * d
     rate = cd / (kms[-1] * 1e-3)
-    peak = SM_COUNT * ALU_LANES * NOMINAL_SM_MHZ * 1e6
+    peak = peak or alu_peak_ops()
     return {"workload": f"{'self' if self_join else 'AB'}-join d={d} n={n} m={m}", "precision": prec,
             "band": [r, W], "band_cell_dims": cd, "main_kernel_ms": kms[-1],
             "computed_cell_dims_per_s": rate, "alu_frac": rate * alu_ops_mode(d, self_join, prec) / peak,
@@ -374,13 +390,13 @@ def main():
         cells0 = computed_cells(n, e, self_join)
         for prec, v in per_prec.items():  # ALU roofline fraction of the main kernel per mode
             rate = cells0 * d / (v["main_kernel_ms"] * 1e-3)
-            v["alu_frac"] = rate * alu_ops_mode(d, self_join, prec) / (SM_COUNT * ALU_LANES * NOMINAL_SM_MHZ * 1e6)
+            v["alu_frac"] = rate * alu_ops_mode(d, self_join, prec) / alu_peak_ops((clocks or {}).get("sm_mhz"))
 
     per_cfg = {}
     if not args.no_per_config and world == 1:
         for name, prec in (("C3", "fp32"), ("C3", "mixed"), ("C3", "fp16"), ("C4", "fp32"), ("C4", "mixed"),
                            ("C4", "fp64"), ("C5", "fp32"), ("C5", "mixed"), ("C5", "fp16"), ("C5", "fp64")):
-            per_cfg[f"{name}/{prec}"] = band_probe(ctx, torch, dev, name, prec)
+            per_cfg[f"{name}/{prec}"] = band_probe(ctx, torch, dev, name, prec, peak=alu_peak_ops((clocks or {}).get("sm_mhz")))
         _PROBE_CACHE.clear()
         torch.cuda.empty_cache()
 
@@ -415,15 +431,18 @@ def main():
             _, bc = mstamp.plan_bands(d, n, m, args.precision, e, self_join, world)
             band_cells = int(bc[0])
         ops = alu_ops_per_cell_dim(d, self_join) * band_cells * d
-        peak_tops = SM_COUNT * ALU_LANES * NOMINAL_SM_MHZ * 1e6 / 1e12
+        lanes, lsrc = alu_lanes()
+        run_mhz = (clocks or {}).get("sm_mhz") or NOMINAL_SM_MHZ
+        peak_tops = alu_peak_ops(run_mhz) / 1e12
         achieved = ops / (kms * 1e-3) / 1e12 if kms > 0 else None
         roof = {"bound": "alu", "achieved": achieved, "peak": peak_tops, "unit": "Tops/s",
                 "frac": achieved / peak_tops if achieved else None,
                 "traffic": load_traffic(args.config, args.precision),
                 "kernel": "mp_diag", "ops_per_cell_dim": alu_ops_per_cell_dim(d, self_join),
                 "computed_cell_dims": band_cells * d,
-                "peak_basis": f"148 SM x 64 ALU lanes/clk x {NOMINAL_SM_MHZ:.0f} MHz (derived; MEASURED_PEAKS {src} "
-                              "has no ALU figure)"}
+                "peak_basis": f"{SM_COUNT} SM x {lanes:.2f} FMNMX lanes/SM/clk ({lsrc}: scripts/pipe_peaks.cu -> "
+                              f"profiles/r1_pipe_peaks.json; MEASURED_PEAKS {src} has no ALU figure) x {run_mhz:.0f} MHz "
+                              "(SM clock sampled during the timed region)"}
         cpu = None
         if not args.no_cpu_baseline and world == 1:
             v, nr, dt, th = oracle_sample(cfg, target_s=args.ref_seconds)
