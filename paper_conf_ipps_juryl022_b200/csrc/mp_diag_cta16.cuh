@@ -35,8 +35,8 @@
 
 namespace mpk {
 
-// Per lane-group-size launch shape (measured on one B200, Mixed, n*d^... self-joins of
-// d = 64 / 128 / 256): warps per block and steps per staging batch (one block barrier per
+// Per lane-group-size launch shape (measured on one B200, Mixed self-joins of d = 64 / 128 / 256,
+// n = 32768 / 16384 / 8192): warps per block and steps per staging batch (one block barrier per
 // batch).  d = 64: 4 warps, SB = 2 (61.0 -> 58.9 ms); d = 128: 8 warps (45.7 -> 39.5 ms);
 // d = 256: 4 warps, SB = 1 (SB = 2: 31.3 -> 34.9 ms, 8 warps: 33.7 ms).
 template <int G> struct CtaShapeH {
