@@ -269,6 +269,17 @@ mp_diag64f(const MainParams p) {
 #pragma unroll
                 for (int kk = 0; kk < DL; ++kk) S[kk] = INF;
             }
+            // ranks some lane can improve (one warp OR; the staged thresholds only decrease, so
+            // this is a superset): the loop below skips the others without any vote
+            unsigned rk_bits = 0;
+#pragma unroll
+            for (int kk = 0; kk < DL; ++kk) {
+                const int pl = kk * G + g;
+                bool hk = S[kk] <= (double)rowv[pl * PSR + sr].thr;
+                if (SELF) hk |= S[kk] <= (double)colv[pl * PSC + sc].thr;
+                rk_bits |= (unsigned)hk << kk;
+            }
+            rk_bits = __reduce_or_sync(FULL, rk_bits);
             // Eq. (3), write-through: rank by rank (S rotates through S[0], so no dynamic
             // register indexing), group min by shuffles, the lowest-index leader merges
             // (value, index) into the global key and lowers the ring threshold
@@ -278,6 +289,7 @@ mp_diag64f(const MainParams p) {
                 const double v = S[0];
 #pragma unroll
                 for (int q = 0; q + 1 < DL; ++q) S[q] = S[q + 1];
+                if (((rk_bits >> kk) & 1u) == 0u) continue;
                 const int rk = rank_of_plane<DL, G>(pl);
                 const bool need_r = __any_sync(FULL, v <= (double)rowv[pl * PSR + sr].thr);
                 const bool need_c = SELF && __any_sync(FULL, v <= (double)colv[pl * PSC + sc].thr);
