@@ -201,6 +201,49 @@ def _half_stats(P_or, I_or, P, I, m):
                 max_rel=float(rel.max()), recall=float((I == I_or)[fin].mean()))
 
 
+@pytest.mark.parametrize("prec", ["fp64", "fp32"])
+@pytest.mark.parametrize("shape", [(3, 1500, 1024, 256, 81), (16, 900, 600, 150, 82), (70, 400, 300, 75, 83)])
+def test_long_windows(ctx, oracle_mod, prec, shape):
+    """Long windows (m up to 1024, the re-seed interval clamped below 8m; seeds of m terms with
+    compensated sums), small and large d, against the oracle at the north-star tolerances."""
+    d, n, m, e, seed = shape
+    T = datagen.random_walk(d, n, m, seed)
+    P, I, P2 = oracle_mod.mstamp(T, m, e)
+    Pg, Ig = ctx.compute(T, m, prec, e)
+    st = parity.check(oracle_mod, T, m, P, I, P2, Pg, Ig, prec)
+    print(prec, shape, st)
+
+
+@pytest.mark.parametrize("prec", ["fp16", "mixed", "fp16c"])
+def test_half_modes_ab_d16(ctx, prec):
+    """AB-join in the half modes at d = 16 (warp half kernel, pairs starting at column -1):
+    error vs the GPU FP64 result (oracle-checked elsewhere) within the stated bound, planted
+    motif recovered, band partials merge bit-identically."""
+    from paper_conf_ipps_juryl022_b200 import mstamp
+    d, n, m = 16, 2000, 64
+    Tq, Tr = datagen.random_walk_ab(d, n, m, 84)
+    Pg, Ig = ctx.compute(Tq, m, prec, Tr=Tr)
+    P64, I64 = ctx.compute(Tq, m, "fp64", Tr=Tr)
+    st = _half_stats(P64, I64, Pg, Ig, m)
+    print(prec, "ab d16", st)
+    assert st["median_rel"] < (0.02 if prec != "fp16" else 0.2)
+    a, b = datagen.motif_positions(n, m)
+    for k in range(d // 2):
+        assert abs(int(Ig[k, a]) - b) <= (0 if prec == "mixed" else m // 16)
+    Td, Trd = torch.from_numpy(Tq).cuda(), torch.from_numpy(Tr).cuda()
+    kw = mstamp.key_words(d, n, prec)
+    full = torch.empty(kw, dtype=torch.int64, device="cuda")
+    ctx.partial_device(Td, m, full, 0, 1, prec, 0, Tr=Trd)
+    parts = []
+    for r in range(4):
+        k = torch.empty(kw, dtype=torch.int64, device="cuda")
+        ctx.partial_device(Td, m, k, r, 4, prec, 0, Tr=Trd)
+        parts.append(k)
+    merged = torch.stack(parts).min(dim=0).values
+    torch.cuda.synchronize()
+    assert torch.equal(merged, full)
+
+
 def test_compute_out_buffers(ctx):
     """Context.compute(out=) (preallocated, e.g. pinned, host outputs: the bench's e2e leg)
     returns exactly what the allocating call returns; malformed outputs are rejected."""
