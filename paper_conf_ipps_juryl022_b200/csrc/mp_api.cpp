@@ -187,11 +187,12 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     const bool half = prec == MP_FP16 || prec == MP_MIXED || prec == MP_FP16C;
     const size_t sb = half ? 16 : 4 * eb;                                   // stats entry bytes
     const size_t tb = prec == MP_FP64 ? 8 : ((prec == MP_FP16 || prec == MP_FP16C) ? 2 : 4);  // precalc value bytes
+    const size_t tbs = prec == MP_FP32 ? 8 : tb;  // window stats scratch (FP32 mode: FP64 precalc, reading R1')
     const mpk::Variant var = mpk::pick_variant(prec, (int)d);
     const int Dp = var.DL * var.G;
     mpk::PreParams pp{};
     pp.n = n; pp.d = (int)d; pp.m = (int)m; pp.Dp = Dp;
-    MP_CUDA(ctx, ensure(ctx->nrm, (size_t)n * d * tb));
+    MP_CUDA(ctx, ensure(ctx->nrm, (size_t)n * d * tbs));
     pp.nrm32 = (float*)ctx->nrm.p; pp.nrm64 = (double*)ctx->nrm.p;
     if (half) {
         MP_CUDA(ctx, ensure(ctx->scale, (size_t)d * sizeof(double)));
@@ -205,7 +206,7 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
         Buf** B = series_bufs[sidx];
         MP_CUDA(ctx, ensure(*B[0], (size_t)n * d * sb));
         if (half) MP_CUDA(ctx, ensure(*B[1], (size_t)(n + 1) * d * sb));  // pair format: n+1 entries
-        MP_CUDA(ctx, ensure(*B[2], (size_t)n * d * tb));
+        MP_CUDA(ctx, ensure(*B[2], (size_t)n * d * tbs));
         MP_CUDA(ctx, ensure(*B[3], (size_t)n * Dp * tb));
         MP_CUDA(ctx, ensure(*B[4], (size_t)L * Dp * tb));
         pp.T = sidx == 0 ? dT : dTr;

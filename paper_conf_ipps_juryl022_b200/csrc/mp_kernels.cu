@@ -46,7 +46,7 @@ __global__ void pre_stats(const PreParams p) {
     if constexpr (sizeof(T) == 4) p.nrm32[(long long)dim * n + pos] = nr; else p.nrm64[(long long)dim * n + pos] = nr;
 }
 
-template <class T>
+template <class T, class A = T>  // A: precalc arithmetic (FP32 mode: FP64, reading R1)
 __global__ void pre_diff(const PreParams p) {
     using V4 = typename PT<T>::V4;
     const long long n = p.n;
@@ -57,25 +57,25 @@ __global__ void pre_diff(const PreParams p) {
     const long long pos = gid / d;  // position-major output
     const int dim = (int)(gid % d);
     const double* x = p.T + (long long)dim * L;
-    const T* mu = reinterpret_cast<const T*>(p.mu) + (long long)dim * n;
-    T nr;
-    if constexpr (sizeof(T) == 4) nr = p.nrm32[(long long)dim * n + pos]; else nr = p.nrm64[(long long)dim * n + pos];
+    const A* mu = reinterpret_cast<const A*>(p.mu) + (long long)dim * n;
+    A nr;
+    if constexpr (sizeof(A) == 4) nr = p.nrm32[(long long)dim * n + pos]; else nr = p.nrm64[(long long)dim * n + pos];
     V4 v;
     if (pos == 0) {
         v.x = 0; v.y = 0;
     } else {
-        const T xl = (T)x[pos + m - 1], xf = (T)x[pos - 1];
-        v.x = (xl - xf) / (T)2;
-        v.y = (xl - mu[pos]) + (xf - mu[pos - 1]);
+        const A xl = (A)x[pos + m - 1], xf = (A)x[pos - 1];
+        v.x = (T)((xl - xf) / (A)2);
+        v.y = (T)((xl - mu[pos]) + (xf - mu[pos - 1]));
     }
-    v.z = nr > (T)0 ? sqrt((T)(2 * m)) / nr : (T)0;
+    v.z = nr > (A)0 ? (T)(sqrt((A)(2 * m)) / nr) : (T)0;
     v.w = 0;
     reinterpret_cast<V4*>(p.st)[pos * d + dim] = v;
 }
 
 // position-major, zero-padded copies of the working-precision series and window means
 // (the seeds' operands: a lane's dims are contiguous, so they load as vectors)
-template <class T>
+template <class T, class A = T>
 __global__ void pre_pm(const PreParams p) {
     const long long n = p.n, L = p.n + p.m - 1;
     const int d = p.d, Dp = p.Dp;
@@ -86,7 +86,7 @@ __global__ void pre_pm(const PreParams p) {
     T* tw = reinterpret_cast<T*>(p.tw);
     T* mup = reinterpret_cast<T*>(p.mup);
     tw[gid] = dim < d ? (T)p.T[(long long)dim * L + t] : (T)0;
-    if (t < n) mup[gid] = dim < d ? reinterpret_cast<const T*>(p.mu)[(long long)dim * n + t] : (T)0;
+    if (t < n) mup[gid] = dim < d ? (T)reinterpret_cast<const A*>(p.mu)[(long long)dim * n + t] : (T)0;
 }
 
 // ------------------------------------------------------------------ precompute, FP16 / Mixed
@@ -481,9 +481,12 @@ cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s) {
         pre_diff<double><<<grid1d(cnt, 256), 256, 0, s>>>(p);
         pre_pm<double><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
     } else if (prec == P32) {
-        pre_stats<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-        pre_diff<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-        pre_pm<float><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
+        // FP32 mode: window stats and df / dg / a in FP64 from the FP64 input, rounded once to
+        // FP32 (reading R1'): FP32 cancellation in x - mu grows with the window's offset.
+        // (FP64 seeds from the FP64 series were measured too: no accuracy gain, C2 +11 %.)
+        pre_stats<double><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+        pre_diff<float, double><<<grid1d(cnt, 256), 256, 0, s>>>(p);
+        pre_pm<float, double><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
     } else {
         const bool mixed = prec == PMIX;
         cudaMemsetAsync(p.maxbits, 0, 2 * p.d * sizeof(unsigned long long), s);

@@ -6,13 +6,20 @@ import os
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
 from paper_conf_ipps_juryl022_b200 import datagen, mstamp  # noqa: E402
+sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
+import parity  # noqa: E402
 
 name, prec = sys.argv[1], sys.argv[2]
 hs = [int(v) for v in sys.argv[3].split(",")]
-cfg = datagen.make(name)
+if name.startswith("X"):   # X<d>_<n>_<m>: ad-hoc self-join shape
+    d_, n_, m_ = (int(v) for v in name[1:].split("_"))
+    cfg = dict(T=datagen.random_walk(d_, n_, m_, 7), Tr=None, d=d_, n=n_, m=m_, exclusion=m_ // 4)
+else:
+    cfg = datagen.make(name)
 d, n, m, e = cfg["d"], cfg["n"], cfg["m"], cfg["exclusion"]
 T = torch.from_numpy(cfg["T"]).cuda()
 Tr = None if cfg["Tr"] is None else torch.from_numpy(cfg["Tr"]).cuda()
@@ -30,8 +37,14 @@ for h in hs:
     for _ in range(3):
         ctx.compute_device(T, m, P, I, prec, e, Tr=Tr)
         torch.cuda.synchronize()
-        ts.append(ctx.last_timing())
+        ts.append(ctx.last_timing()[0])
     ok = torch.isfinite(P0) & (P0 > 1e-6)
     err = ((P - P0).abs()[ok] / P0[ok]).max().item()
+    # error in units of the parity tolerance (tests/parity.py; FP64 GPU result as reference)
+    p0 = P0.cpu().numpy()
+    fin = np.isfinite(p0)
+    tol = parity.tol_of(np.where(fin, p0, 0.0), m, "fp64" if prec == "fp64" else "fp32",
+                        P0_row=np.where(fin[0], p0[0], np.inf))
+    ratio = float((np.abs(np.where(fin, P.cpu().numpy() - p0, 0.0)) / tol).max())
     same_i = (I == I0).float().mean().item()
-    print(f"{name} {prec} H={h} main_ms={min(ts):.2f} max_rel_err={err:.3e} idx_agree={same_i:.4f}", flush=True)
+    print(f"{name} {prec} H={h} main_ms={min(ts):.2f} max_rel_err={err:.3e} idx_agree={same_i:.4f} err/tol={ratio:.3f}", flush=True)
