@@ -62,7 +62,8 @@ typedef struct mp_ctx mp_ctx;   /* opaque */
 typedef struct {
     int device;             /* CUDA device ordinal this context drives (one process per GPU) */
     int64_t reseed_h[4];    /* re-seed interval H (rows) for FP64, FP32, FP16 (also FP16C), MIXED;
-                               0 -> default (R2) */
+                               0 -> default (R2); rounded up to a multiple of 8 (re-seeds
+                               fall on staging-batch starts); < 0 or > 2^30 -> MP_ERR_INVALID */
 } mp_config;
 
 /* Create a context on cfg->device (cfg == NULL -> device 0, defaults). */

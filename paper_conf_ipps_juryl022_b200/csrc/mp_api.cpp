@@ -170,7 +170,11 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     const bool self = dTr == nullptr;
     const int64_t L = n + m - 1;
     const size_t eb = elt_bytes(prec);
-    const int64_t H = ctx->H[prec] > 0 ? ctx->H[prec] : default_h(prec, m);
+    // re-seeds happen at staging-batch starts (every kernel steps in batches of 1, 2 or 4 rows),
+    // so the interval is rounded up to a multiple of 8: then every re-seed row i = 0 mod H is a
+    // batch start in every kernel variant (include/mp.h, mp_config.reseed_h)
+    int64_t H = ctx->H[prec] > 0 ? ctx->H[prec] : default_h(prec, m);
+    H = std::min<int64_t>((H + 7) / 8 * 8, int64_t(1) << 30);
     if (self && excl < 0) excl = (m + 3) / 4;
 
     // flag non-finite inputs (reading G23)
@@ -192,6 +196,7 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     const int Dp = var.DL * var.G;
     mpk::PreParams pp{};
     pp.n = n; pp.d = (int)d; pp.m = (int)m; pp.Dp = Dp;
+    if (var.ctab) { pp.pm_G = var.G; pp.pm_DL = var.DL; }
     MP_CUDA(ctx, ensure(ctx->nrm, (size_t)n * d * tbs));
     pp.nrm32 = (float*)ctx->nrm.p; pp.nrm64 = (double*)ctx->nrm.p;
     if (half) {
@@ -315,7 +320,7 @@ mp_status mp_init(mp_ctx** out, const mp_config* cfg) {
         ctx->H[4] = cfg->reseed_h[2];  // FP16C follows FP16
     }
     for (int i = 0; i < 5; ++i)
-        if (ctx->H[i] < 0) { delete ctx; return MP_ERR_INVALID; }
+        if (ctx->H[i] < 0 || ctx->H[i] > (int64_t(1) << 30)) { delete ctx; return MP_ERR_INVALID; }
     int ndev = 0;
     cudaError_t e = cudaGetDeviceCount(&ndev);
     if (e != cudaSuccess || ndev == 0) { delete ctx; return MP_ERR_CUDA; }

@@ -54,6 +54,9 @@
 #ifndef MP_KEEP_DL
 #define MP_KEEP_DL 16
 #endif
+#ifndef MP_FOLD
+#define MP_FOLD 4   // steps between the Fast2Sum folds of the compensated QT (power of two)
+#endif
 #ifndef MP_SEED_CHUNK
 #define MP_SEED_CHUNK 4
 #endif
@@ -79,6 +82,9 @@ constexpr unsigned DIRTY = 0x80000000u;
 template <class T> struct PT;
 template <> struct PT<float> {
     using V4 = float4;
+    // 'a' of padded dimensions / positions: D = sqrt(|2m - QT a a|) ~ 1e18 sorts last; finite,
+    // so the compensated evaluation fma(-QT_lo, a a, .) never forms 0 * inf
+    static __device__ __forceinline__ float pad_a() { return 1e18f; }
     static __device__ __forceinline__ float inf() { return __int_as_float(0x7f800000); }
     static __device__ __forceinline__ float ninf() { return __int_as_float(0xff800000); }
     // sqrt of |x|: |x| absorbs the rounding residue of 2m - QT a_i a_j near D = 0
@@ -94,6 +100,7 @@ template <> struct PT<float> {
 };
 template <> struct PT<double> {
     using V4 = double4;
+    static __device__ __forceinline__ double pad_a() { return 1e18; }
     static __device__ __forceinline__ double inf() { return __longlong_as_double(0x7ff0000000000000ll); }
     static __device__ __forceinline__ double ninf() { return __longlong_as_double((long long)0xfff0000000000000ull); }
     static __device__ __forceinline__ double sqrt_abs(double x) { return sqrt(fabs(x)); }  // IEEE RN
@@ -288,10 +295,11 @@ constexpr long long EXT_EMPTY = 0x7FFFFFFFFFFFFFFFll;                  // INT64_
 template <class T> struct KeyOps;
 template <> struct KeyOps<float> {
     using K = unsigned long long;
-    // async-stage the key's value (high word) into thr and its index (low word) into idx
-    static __device__ __forceinline__ void stage(const K* p, float* thr, unsigned* idx) {
+    // async-stage the key's value (high word) into the threshold hint thr and the whole key
+    // (one 8-byte copy: value and index always from the same atomicMin state) into key
+    static __device__ __forceinline__ void stage(const K* p, float* thr, K* key) {
         cp_async4(thr, reinterpret_cast<const char*>(p) + 4);
-        cp_async4(idx, p);
+        cp_async8(key, p);
     }
     static __device__ __forceinline__ void merge(K* p, float v, unsigned i) {
         atomicMin(p, ((K)__float_as_uint(v) << 32) | (K)i);
@@ -413,7 +421,7 @@ template <class T, int DL, int G, int W> struct Smem {
     using Gm = Geo<G, W>;
     static constexpr int D = DL * G;
     static constexpr size_t ring_bytes =
-        (((size_t)D * (Gm::PSR + Gm::PSC) * (sizeof(V4) + sizeof(unsigned))) + 15) & ~(size_t)15;
+        (((size_t)D * (Gm::PSR + Gm::PSC) * (sizeof(V4) + sizeof(typename KeyOps<T>::K))) + 15) & ~(size_t)15;
     static constexpr size_t flag_bytes = 0;  // dirty flags live in registers (bit masks)
     static constexpr size_t bytes_per_warp = ring_bytes + flag_bytes + (size_t)W * DL * 32 * sizeof(T);
     // warps per block: up to 4, fewer when a warp's rings are large (blocks <= ~112 KB)
@@ -441,14 +449,17 @@ mp_diag(const MainParams p) {
     constexpr int CA = Gm::CA, RA = Gm::RA, CW = Gm::CW, D = DL * G;
     constexpr int PSR = Gm::PSR, PSC = Gm::PSC;
     constexpr int SB = Gm::SB;
+    constexpr int FOLD = SB > MP_FOLD ? SB : MP_FOLD;  // steps between folds of QL into QT
 
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     unsigned char* wbase = smem_raw + (size_t)warp * SM::bytes_per_warp;
     V4* rowv = reinterpret_cast<V4*>(wbase);
     V4* colv = rowv + (size_t)D * PSR;
-    unsigned* rowi = reinterpret_cast<unsigned*>(colv + (size_t)D * PSC);
-    unsigned* coli = rowi + (size_t)D * PSR;
+    // ring keys: the warp's current (value, index) best of each staged (position, rank), the
+    // index word's bit 31 marking it dirty; the .w words are filter hints only
+    K* rowi = reinterpret_cast<K*>(colv + (size_t)D * PSC);
+    K* coli = rowi + (size_t)D * PSR;
     // dirty ring slots: warp-uniform bit masks in registers (slot -> bit), set after each
     // slow path by a warp OR-reduction, cleared on eviction -- no shared-memory flags to poll
     static_assert(Gm::RING_R <= 64 && Gm::RING_C <= 64, "dirty masks hold one bit per ring slot");
@@ -488,7 +499,7 @@ mp_diag(const MainParams p) {
         const int cnt = p_hi - p_lo;
         if (cnt <= 0) return;
         V4* buf = is_row ? rowv : colv;
-        unsigned* ib = is_row ? rowi : coli;
+        K* ib = is_row ? rowi : coli;
         const int ps = is_row ? PSR : PSC;
         const V4* __restrict__ st = is_row ? st_q : st_r;
         const bool want_thr = is_row || SELF;
@@ -526,15 +537,15 @@ mp_diag(const MainParams p) {
                     cp_async16(dst, src);
                     cp_async8(&dst->z, &src->z);
                 }
-            } else {  // padded dimension: a = +inf with QT = -1 gives D = +inf (sorts last)
-                dst->x = 0; dst->y = 0; dst->z = INF;
+            } else {  // padded dimension: a = pad_a with QT = -1 gives D ~ 1e18 (sorts last)
+                dst->x = 0; dst->y = 0; dst->z = PT<T>::pad_a();
             }
             const int rk = rank_of_plane<DL, G>(pl);
             if (rk < d && want_thr) {
                 KO::stage(keys + (size_t)pos * d + rk, &dst->w, &ib[pl * ps + sl]);
             } else {
                 dst->w = NINF;  // never hit
-                ib[pl * ps + sl] = 0x7fffffffu;
+                ib[pl * ps + sl] = EMPTY32;
             }
         }
     };
@@ -543,7 +554,7 @@ mp_diag(const MainParams p) {
         const int cnt = p_hi - p_lo;
         if (cnt <= 0) return;
         const V4* buf = is_row ? rowv : colv;
-        const unsigned* ib = is_row ? rowi : coli;
+        const K* ib = is_row ? rowi : coli;
         const int ps = is_row ? PSR : PSC;
         // early out (warp-uniform, registers only): most evictions find nothing dirty
         DMask& dm = is_row ? dmask_r : dmask_c;
@@ -564,8 +575,8 @@ mp_diag(const MainParams p) {
             if (((dirty >> sl) & 1ull) == 0) continue;
             const int rk = rank_of_plane<DL, G>(pl);
             if (rk >= d) continue;
-            const unsigned ix = ib[pl * ps + sl];
-            if (ix & DIRTY) KO::merge(keys + (size_t)pos * d + rk, buf[pl * ps + sl].w, ix & ~DIRTY);
+            const K kv = ib[pl * ps + sl];
+            if (kv & DIRTY) atomicMin(keys + (size_t)pos * d + rk, kv & ~(K)DIRTY);
         }
     };
 
@@ -598,7 +609,9 @@ mp_diag(const MainParams p) {
         // (Kahan) accumulation, at each cell's first row and then every H rows (reseed(),
         // called at warp-uniform steps; the tile is HT >= H rows tall).  Operands are
         // position-major and padded to D dims, so a lane (G == 1) loads its DL dims as vectors.
-        T QT[W][DL];
+        // QT = QT[u][kk] + QL[u][kk] (compensated, reading R4): increments accumulate into the
+        // small word QL, which is folded into QT by an exact Fast2Sum every FOLD steps
+        T QT[W][DL], QL[W][DL];
         auto seed_cell = [&](int u, long long row) {
             // dims in chunks of SC: the m-long dot-product loop then keeps few operand
             // registers live, so seeding never sets the kernel's register peak
@@ -627,8 +640,11 @@ mp_diag(const MainParams p) {
                     }
                 }
 #pragma unroll
-                for (int kk = 0; kk < SC; ++kk)
-                    QT[u][c0 + kk] = ((c0 + kk) * G + g) >= d ? (T)-1 : acc[kk];  // padded dims: zero data
+                for (int kk = 0; kk < SC; ++kk) {  // the Kahan sum is acc - cmp: keep both words
+                    const bool pad = ((c0 + kk) * G + g) >= d;  // padded dims: zero data
+                    QT[u][c0 + kk] = pad ? (T)-1 : acc[kk];
+                    QL[u][c0 + kk] = pad ? (T)0 : -cmp[kk];
+                }
             }
         };
 #pragma unroll
@@ -637,7 +653,7 @@ mp_diag(const MainParams p) {
                 seed_cell(u, lo[u]);
             } else {
 #pragma unroll
-                for (int kk = 0; kk < DL; ++kk) QT[u][kk] = (kk * G + g) >= d ? (T)-1 : (T)0;
+                for (int kk = 0; kk < DL; ++kk) { QT[u][kk] = (kk * G + g) >= d ? (T)-1 : (T)0; QL[u][kk] = (T)0; }
             }
         }
         int seeded_step = -1;  // step whose row was re-seeded at its batch start
@@ -693,13 +709,15 @@ mp_diag(const MainParams p) {
                 const V4 C = colv[pl * PSC + scn];
                 if constexpr (W == 2) {
                     const V4 C0v = Cold[kk];
-                    if (upd[0]) QT[0][kk] = fma(R.x, C0v.y, fma(C0v.x, R.y, QT[0][kk]));   // Eq. (1)
-                    S[0][kk] = PT<T>::sqrt_abs(fma(-QT[0][kk], R.z * C0v.z, two_m));
+                    if (upd[0]) QL[0][kk] = fma(R.x, C0v.y, fma(C0v.x, R.y, QL[0][kk]));   // Eq. (1)
+                    const T pr0 = R.z * C0v.z;
+                    S[0][kk] = PT<T>::sqrt_abs(fma(-QL[0][kk], pr0, fma(-QT[0][kk], pr0, two_m)));
                     if constexpr (KEEP) tc0[kk] = C0v.w;
                     Cnew[kk] = C;
                 }
-                if (upd[W - 1]) QT[W - 1][kk] = fma(R.x, C.y, fma(C.x, R.y, QT[W - 1][kk]));
-                S[W - 1][kk] = PT<T>::sqrt_abs(fma(-QT[W - 1][kk], R.z * C.z, two_m));  // Eq. (1)
+                if (upd[W - 1]) QL[W - 1][kk] = fma(R.x, C.y, fma(C.x, R.y, QL[W - 1][kk]));  // Eq. (1)
+                const T pr = R.z * C.z;
+                S[W - 1][kk] = PT<T>::sqrt_abs(fma(-QL[W - 1][kk], pr, fma(-QT[W - 1][kk], pr, two_m)));  // Eq. (1)
                 if constexpr (KEEP) {
                     tr[kk] = R.w;
                     if constexpr (W == 1) tc0[kk] = C.w;
@@ -794,11 +812,12 @@ mp_diag(const MainParams p) {
                         for (int u = W - 1; u >= 0; --u)
                             if (v[u] == vr) j = col[u];                 // lowest column first
                         const int ix = pl * PSR + sr;
-                        const T cur = rowv[ix].w;
-                        const unsigned ci = rowi[ix] & ~DIRTY;
+                        const K kc = rowi[ix];
+                        const T cur = __uint_as_float((unsigned)(kc >> 32));
+                        const unsigned ci = (unsigned)kc & ~DIRTY;
                         if (vr < cur || (vr == cur && (unsigned)j < ci)) {
                             rowv[ix].w = vr;
-                            rowi[ix] = (unsigned)j | DIRTY;
+                            rowi[ix] = ((K)__float_as_uint(vr) << 32) | (unsigned)j | DIRTY;
                             mark_r |= 1ull << sr;
                         }
                     }
@@ -814,11 +833,12 @@ mp_diag(const MainParams p) {
                             if (vc < INF && eqc != 0 && lane == 31 - __clz(eqc)) {
                                 const int scu = Gm::scol(col[u]);
                                 const int ix = pl * PSC + scu;
-                                const T cur = colv[ix].w;
-                                const unsigned ci = coli[ix] & ~DIRTY;
+                                const K kc = coli[ix];
+                                const T cur = __uint_as_float((unsigned)(kc >> 32));
+                                const unsigned ci = (unsigned)kc & ~DIRTY;
                                 if (vc < cur || (vc == cur && (unsigned)row < ci)) {
                                     colv[ix].w = vc;
-                                    coli[ix] = (unsigned)row | DIRTY;
+                                    coli[ix] = ((K)__float_as_uint(vc) << 32) | (unsigned)row | DIRTY;
                                     mark_c |= 1ull << scu;
                                 }
                             }
@@ -892,6 +912,16 @@ mp_diag(const MainParams p) {
 
         int to_seed = H;  // steps until the next re-seed (H is a multiple of SB)
         for (int s0 = 0; s0 < s_end; s0 += SB) {
+            if ((s0 & (FOLD - 1)) == 0) {  // fold the increments into QT (exact Fast2Sum)
+#pragma unroll
+                for (int u = 0; u < W; ++u)
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) {
+                        const T t = QT[u][kk] + QL[u][kk];
+                        QL[u][kk] = QL[u][kk] - (t - QT[u][kk]);
+                        QT[u][kk] = t;
+                    }
+            }
             // seeds: each cell's first row at s0 = 0, then the current row every H steps
             // (H is a multiple of SB, so re-seeds fall on batch starts: one call site)
             if (s0 > 0 && (to_seed -= SB) == 0) {

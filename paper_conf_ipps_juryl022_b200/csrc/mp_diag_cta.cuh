@@ -60,6 +60,7 @@ mp_diag_cta(const MainParams p) {
     using V4 = float4;
     using K = unsigned long long;
     constexpr int D = Cg::D, NCC = Cg::NCC, RR = Cg::RR, RC = Cg::RC, SS = Cg::SS, SB = Cg::SB, NT = Cg::NT;
+    constexpr int FOLD = SB > MP_FOLD ? SB : MP_FOLD;  // steps between folds of QL into QT
 
     extern __shared__ __align__(16) unsigned char smem_raw[];
     V4* rowv = reinterpret_cast<V4*>(smem_raw);
@@ -112,8 +113,8 @@ mp_diag_cta(const MainParams p) {
                 const V4* src = st + (size_t)pos * d + pl;
                 cp_async8(dst, src);
                 cp_async4(&dst->z, &src->z);
-            } else {  // padded dimension / position past the end: D = +inf, never hit
-                dst->x = 0.f; dst->y = 0.f; dst->z = __int_as_float(0x7f800000);
+            } else {  // padded dimension / position past the end: D ~ 1e18 (sorts last), never hit
+                dst->x = 0.f; dst->y = 0.f; dst->z = PT<float>::pad_a();
             }
             if (pos >= 0 && pos < n32 && rk < d && want_thr) {
                 const K* ks = keys + (size_t)pos * d + rk;
@@ -165,7 +166,8 @@ mp_diag_cta(const MainParams p) {
         if (delta > p.delta_hi) hi = lo;
         const int lo32 = (int)lo, hi32 = (int)hi, dlt = (int)delta;
 
-        float QT[DL];
+        // QT = QT[kk] + QL[kk] (compensated, reading R4; see mp_diag)
+        float QT[DL], QL[DL];
         auto seed_cell = [&](long long row) {  // direct centred dot product, compensated
             constexpr int SC = (DL % MP_SEED_CHUNK == 0) ? MP_SEED_CHUNK : DL;
             const long long i0 = row, j0 = row + delta;
@@ -192,15 +194,18 @@ mp_diag_cta(const MainParams p) {
                     }
                 }
 #pragma unroll
-                for (int kk = 0; kk < SC; ++kk)
-                    QT[c0 + kk] = ((c0 + kk) * G + g) >= d ? -1.f : acc[kk];
+                for (int kk = 0; kk < SC; ++kk) {  // the Kahan sum is acc - cmp: keep both words
+                    const bool pad = ((c0 + kk) * G + g) >= d;
+                    QT[c0 + kk] = pad ? -1.f : acc[kk];
+                    QL[c0 + kk] = pad ? 0.f : -cmp[kk];
+                }
             }
         };
         if (lo < hi) {
             seed_cell(lo);
         } else {
 #pragma unroll
-            for (int kk = 0; kk < DL; ++kk) QT[kk] = (kk * G + g) >= d ? -1.f : 0.f;
+            for (int kk = 0; kk < DL; ++kk) { QT[kk] = (kk * G + g) >= d ? -1.f : 0.f; QL[kk] = 0.f; }
         }
 
         const int nrows = (int)(r1 - r0);
@@ -215,6 +220,14 @@ mp_diag_cta(const MainParams p) {
         int seeded_step = -1;
         int to_seed = H;
         for (int s0 = 0; s0 < nrows; s0 += SB) {
+            if ((s0 & (FOLD - 1)) == 0) {  // fold the increments into QT (exact Fast2Sum)
+#pragma unroll
+                for (int kk = 0; kk < DL; ++kk) {
+                    const float t = QT[kk] + QL[kk];
+                    QL[kk] = QL[kk] - (t - QT[kk]);
+                    QT[kk] = t;
+                }
+            }
             if (s0 > 0 && (to_seed -= SB) == 0) {
                 to_seed = H;
                 const long long row = R0 + s0;
@@ -246,8 +259,9 @@ mp_diag_cta(const MainParams p) {
                     const int pl = kk * G + g;
                     const V4 R = rowv[sr * SS + pl];
                     const V4 C = colv[sc * SS + pl];
-                    if (upd) QT[kk] = fmaf(R.x, C.y, fmaf(C.x, R.y, QT[kk]));          // Eq. (1)
-                    S[kk] = PT<float>::sqrt_abs(fmaf(-QT[kk], R.z * C.z, two_m));      // Eq. (1)
+                    if (upd) QL[kk] = fmaf(R.x, C.y, fmaf(C.x, R.y, QL[kk]));          // Eq. (1)
+                    const float pr = R.z * C.z;
+                    S[kk] = PT<float>::sqrt_abs(fmaf(-QL[kk], pr, fmaf(-QT[kk], pr, two_m)));  // Eq. (1)
                 }
                 sort_net<float, DL>(S);                                               // Eq. (2)
                 if constexpr (MP_FUSE_LAST && G > 1) {

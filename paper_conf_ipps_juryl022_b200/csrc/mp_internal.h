@@ -41,6 +41,8 @@ struct PreParams {
     void* mu;           // out window mean [dim][pos]
     void* mup;          // out window mean, position-major padded [pos][Dp] (seeds)
     int Dp;             // padded dimension count of the kernel variant (DL * G)
+    int pm_G, pm_DL;    // pm_G > 0: the seed operands (tw, mup) store dim kk*G + g at g*DL + kk, so
+                        // each lane's DL dims are contiguous (mp_diag_ctab); 0: natural order
     float* nrm32;       // scratch for FP32 path (norm) [dim][pos]
     double* nrm64;
     long long n;
@@ -56,7 +58,8 @@ struct PreParams {
 enum { P64 = 0, P32 = 1, P16 = 2, PMIX = 3, P16C = 4 };
 
 // Variant selection for a given (precision, d): dims per lane DL and lanes per cell G.
-struct Variant { int DL; int G; int W; int NC; int cta = 0; /* warps per block of the block-cooperative kernel, 0: warp tiles */ };
+struct Variant { int DL; int G; int W; int NC; int cta = 0; /* warps per block of the block-cooperative kernel, 0: warp tiles */
+                 bool ctab = false; /* FP32 block-cooperative kernel with TMA staging (mp_diag_ctab) */ };
 Variant pick_variant(int prec, int d);
 size_t smem_per_block(int prec, int d, bool self);
 int variant_warps_per_block(int prec, int d, bool self);

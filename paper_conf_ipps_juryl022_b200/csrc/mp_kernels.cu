@@ -6,6 +6,7 @@
 #include "mp_diag_cta.cuh"
 #include "mp_diag_cta16.cuh"
 #include "mp_diag_cta64.cuh"
+#include "mp_diag_ctab.cuh"
 
 namespace mpk {
 
@@ -85,8 +86,10 @@ __global__ void pre_pm(const PreParams p) {
     const int dim = (int)(gid % Dp);
     T* tw = reinterpret_cast<T*>(p.tw);
     T* mup = reinterpret_cast<T*>(p.mup);
-    tw[gid] = dim < d ? (T)p.T[(long long)dim * L + t] : (T)0;
-    if (t < n) mup[gid] = dim < d ? (T)reinterpret_cast<const A*>(p.mu)[(long long)dim * n + t] : (T)0;
+    // pm_G > 0: dim kk*G + g is stored at g*DL + kk (each lane's dims contiguous)
+    const long long o = p.pm_G > 0 ? t * Dp + (dim % p.pm_G) * p.pm_DL + dim / p.pm_G : gid;
+    tw[o] = dim < d ? (T)p.T[(long long)dim * L + t] : (T)0;
+    if (t < n) mup[o] = dim < d ? (T)reinterpret_cast<const A*>(p.mu)[(long long)dim * n + t] : (T)0;
 }
 
 // ------------------------------------------------------------------ precompute, FP16 / Mixed
@@ -339,6 +342,7 @@ Variant pick_variant(int prec, int d) {
     } else {
         if (dp <= 8) { v.DL = dp; v.G = 1; v.W = 2; }
         else if (dp == 16) { v.DL = 16; v.G = 1; v.W = 1; if (MP_CTA_NW && dp >= MP_CTA_MIN_DP) v.cta = MP_CTA_NW; }
+        else if (MP_CTAB_ON && dp >= 64) { v.DL = ctab_dl(dp); v.G = dp / v.DL; v.W = 1; v.cta = MP_CTAB_NT / 32; v.ctab = true; }
         else if (dp <= 512) { v.DL = 16; v.G = dp / 16; v.W = 1; if (MP_CTA_NW && dp >= MP_CTA_MIN_DP) v.cta = MP_CTA_NW; }
         else { v.DL = 32; v.G = dp / 32; v.W = 1; }
     }
@@ -414,6 +418,23 @@ static long long dispatch_cta(int op, int G, const MainParams* p, int grid, cuda
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
 }
 
+template <bool SELF>
+static long long dispatch_ctab(int op, int dpad, const MainParams* p, int grid, cudaStream_t s) {
+#define MP_BCASE(dp)                                                                       \
+    if (dpad == dp) {                                                                      \
+        using I = InstCtab<ctab_dl(dp), dp / ctab_dl(dp), MP_CTAB_NT, SELF>;               \
+        if (op == 0) return (long long)I::smem();                                          \
+        if (op == 1) return (long long)I::launch(*p, grid, s);                             \
+        if (op == 3) return 1;  /* one tile per block */                                   \
+        return I::blocks_per_sm();                                                         \
+    }
+#if MP_CTAB_ON
+    MP_BCASE(64) MP_BCASE(128) MP_BCASE(256) MP_BCASE(512) MP_BCASE(1024)
+#endif
+#undef MP_BCASE
+    return op == 1 ? (long long)cudaErrorInvalidValue : 0;
+}
+
 template <bool SELF, int MODE>
 static long long dispatch_ctah(int op, int G, const MainParams* p, int grid, cudaStream_t s) {
 #define MP_HCCASE(g)                                                                       \
@@ -457,6 +478,7 @@ static long long dispatch(int op, int prec, bool self, int d, const MainParams* 
         return self ? dispatch_ctah<true, 2>(op, v.G, p, grid, s) : dispatch_ctah<false, 2>(op, v.G, p, grid, s);
     }
     if (v.cta && prec == P64) return self ? dispatch_cta64<true>(op, v.G, p, grid, s) : dispatch_cta64<false>(op, v.G, p, grid, s);
+    if (v.ctab) return self ? dispatch_ctab<true>(op, v.DL * v.G, p, grid, s) : dispatch_ctab<false>(op, v.DL * v.G, p, grid, s);
     if (v.cta) return self ? dispatch_cta<true>(op, v.G, p, grid, s) : dispatch_cta<false>(op, v.G, p, grid, s);
     if (prec == P16) return self ? dispatch_h<true, 0>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 0>(op, v.DL, v.G, p, grid, s);
     if (prec == PMIX) return self ? dispatch_h<true, 1>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 1>(op, v.DL, v.G, p, grid, s);

@@ -5,52 +5,67 @@ Independent of the oracle's formula: it z-normalises every window explicitly
 normalised windows -- the definition PAPER.md:L469 names ("Z-normalized
 Euclidian distance") -- instead of sqrt(2m(1 - rho)) (Eq. (1)).  The two agree in
 real arithmetic; agreement to ~1e-12 pins the oracle's Eq. (1) arithmetic.
-Flat windows are normalised to all-zeros, which reproduces reading G4 (rho = 0,
-D = sqrt(2m)).
+Reading G4 (a flat window, norm 0, has rho = 0 against everything, so D = sqrt(2m)) is
+applied explicitly: any cell with a flat window on either side gets D = sqrt(2m).  (Plain
+z-normalisation to all-zeros would give sqrt(m) against a non-flat window and 0 between
+two flat ones, which is not G4.)
 """
 import numpy as np
 
 
 def znorm_windows(x, m):
+    """(z-normalised windows, flat mask); flat windows are left as zeros and masked."""
     w = np.lib.stride_tricks.sliding_window_view(x, m)
     mu = w.mean(axis=1, keepdims=True)
     sd = w.std(axis=1, keepdims=True)
     z = np.where(sd > 0, (w - mu) / np.where(sd > 0, sd, 1.0), 0.0)
-    return z
+    return z, sd[:, 0] == 0
 
 
 def dist_cube(T, m, Tr=None):
-    """D[k, i, j] z-normalised Euclidean distances (dense; tiny inputs only)."""
+    """D[k, i, j] z-normalised Euclidean distances (dense; tiny inputs only); G4 for flat windows."""
     Tr = T if Tr is None else Tr
     d = T.shape[0]
     out = []
     for k in range(d):
-        zq = znorm_windows(T[k], m)
-        zr = znorm_windows(Tr[k], m)
+        zq, fq = znorm_windows(T[k], m)
+        zr, fr = znorm_windows(Tr[k], m)
         diff = zq[:, None, :] - zr[None, :, :]
-        out.append(np.sqrt((diff * diff).sum(axis=2)))
+        D = np.sqrt((diff * diff).sum(axis=2))
+        out.append(np.where(fq[:, None] | fr[None, :], np.sqrt(2.0 * m), D))
     return np.stack(out)
 
 
 def mstamp(T, m, exclusion, Tr=None):
-    """Returns P (d,n), I (d,n) by sorting each cell's d distances (Python sorted)."""
+    """Returns P (d,n), I (d,n), P2 (d,n) by sorting each cell's d distances (Python sorted).
+
+    P2[k][i] is the runner-up: the smallest D''_k(i, j) over admissible j other than I[k][i]
+    (so P2 == P when another j ties the minimum exactly); +inf when fewer than two j exist."""
     D = dist_cube(T, m, Tr)
     d, n, _ = D.shape
     P = np.full((d, n), np.inf)
+    P2 = np.full((d, n), np.inf)
     I = np.full((d, n), -1, dtype=np.int64)
     for i in range(n):
+        vals = []
         for j in range(n):
             if Tr is None and abs(i - j) <= exclusion:
                 continue
             s = sorted(D[:, i, j].tolist())
             acc = 0.0
+            row = []
             for k in range(d):
                 acc += s[k]
-                v = acc / (k + 1)
-                if v < P[k, i]:
-                    P[k, i] = v
-                    I[k, i] = j
-    return P, I
+                row.append(acc / (k + 1))
+            vals.append((j, row))
+        for k in range(d):
+            # lowest value, then lowest j (reading G2); the runner-up is the next entry
+            ranked = sorted((row[k], j) for j, row in vals)
+            if ranked:
+                P[k, i], I[k, i] = ranked[0]
+            if len(ranked) > 1:
+                P2[k, i] = ranked[1][0]
+    return P, I, P2
 
 
 def mass_1d(x, m, exclusion, xr=None):

@@ -39,6 +39,8 @@ def test_c1_full(ctx, oracle_mod, c1_oracle, prec):
     Pg, Ig = ctx.compute(cfg["T"], cfg["m"], prec, cfg["exclusion"])
     st = parity.check(oracle_mod, cfg["T"], cfg["m"], P, I, P2, Pg, Ig, prec)
     print(prec, st)
+    # the index rule is only as strong as its strict set: most entries must be decided there
+    assert st["exact_idx"] >= 0.9 * st["count"], st
     a, b = datagen.motif_positions(cfg["n"], cfg["m"])
     for k in range(max(1, cfg["d"] // 2)):
         assert Ig[k, a] == b and Ig[k, b] == a
@@ -80,10 +82,14 @@ def test_golden_m2(ctx):
     """Hand-derived closed-form profile (tests/golden/m2_selfjoin.txt) on the GPU, FP64."""
     import test_oracle
     T, meta, rows = test_oracle._read_golden("m2_selfjoin.txt")
+    m = meta["m"]
     for prec in ("fp64", "fp32"):
-        Pg, Ig = ctx.compute(T, meta["m"], prec, meta["exclusion"])
+        Pg, Ig = ctx.compute(T, m, prec, meta["exclusion"])
         for (i, k, p, ok) in rows:
-            assert abs(Pg[k, i] - p) < 1e-3, (prec, i, k, Pg[k, i], p)
+            # exact zeros come out as sqrt of a rounding residue: the near-exact floor of
+            # tests/parity.py, sqrt(2 m rho_tol) (2e-6 in FP64, 6.3e-3 in FP32)
+            tol = parity.tol_of(np.array([[p]]), m, prec, P0_row=np.array([0.0]))[0, 0]
+            assert abs(Pg[k, i] - p) <= tol, (prec, i, k, Pg[k, i], p, tol)
             assert int(Ig[k, i]) in ok, (prec, i, k, Ig[k, i], ok)
 
 
@@ -113,7 +119,7 @@ def test_reseed_interval_independent(ctx, oracle_mod, prec):
     from paper_conf_ipps_juryl022_b200 import mstamp
     T = datagen.random_walk(4, 3000, 32, 33)
     P, I, P2 = oracle_mod.mstamp(T, 32, 8)
-    for h in (7, 64, 5000):
+    for h in (7, 64, 5000):   # 7 -> 8: intervals are rounded up to a multiple of 8 (include/mp.h)
         c = mstamp.Context(0, reseed_h=[h, h, h, h])
         Pg, Ig = c.compute(T, 32, prec, 8)
         c.close()

@@ -38,20 +38,67 @@ def test_oracle_vs_znormalised_bruteforce(oracle_mod, d, n, m, e, seed):
     """Eq. (1) sqrt(2m(1-rho)) == Euclidean distance of z-normalised windows."""
     T = datagen.random_walk(d, n, m, seed, motif=False)
     P, I, P2 = oracle_mod.mstamp(T, m, e)
-    Pb, Ib = brute.mstamp(T, m, e)
+    Pb, Ib, P2b = brute.mstamp(T, m, e)
     tol = _near_tol(Pb, m, rtol=1e-11)
     fin = np.isfinite(Pb)
     assert np.array_equal(fin, np.isfinite(P))
     assert np.all(np.abs(P[fin] - Pb[fin]) <= tol[fin] + 1e-13)
     _check_index(P, I, P2, Ib, Pb, 1e-9)
+    # the runner-up (the value the index rule of tests/parity.py rests on) against the brute force
+    fin2 = np.isfinite(P2b)
+    assert np.array_equal(fin2, np.isfinite(P2))
+    assert np.all(np.abs(P2[fin2] - P2b[fin2]) <= _near_tol(P2b, m, rtol=1e-11)[fin2] + 1e-13)
 
 
 def test_oracle_ab_join_vs_bruteforce(oracle_mod):
     Tq, Tr = datagen.random_walk_ab(3, 80, 12, 7, motif=False)
     P, I, P2 = oracle_mod.mstamp(Tq, 12, Tr=Tr)
-    Pb, Ib = brute.mstamp(Tq, 12, 0, Tr=Tr)
+    Pb, Ib, P2b = brute.mstamp(Tq, 12, 0, Tr=Tr)
     assert np.allclose(P, Pb, rtol=1e-11, atol=1e-12)
+    assert np.allclose(P2, P2b, rtol=1e-11, atol=1e-12)
     _check_index(P, I, P2, Ib, Pb, 1e-9)
+
+
+def _plant_copies(T, m, src, dsts):
+    """Exact copies of window src at each window start in dsts, in every dimension: the copied
+    windows are bit-identical, so every query ties exactly between them (and src)."""
+    T = T.copy()
+    for x in dsts:
+        T[:, x:x + m] = T[:, src:src + m]
+    return T
+
+
+@pytest.mark.parametrize("ab", [False, True])
+def test_runner_up_with_exact_ties(oracle_mod, ab):
+    """Runner-up P2 (the oracle's best2, Eq. (3) L538-549 + reading G2) against the brute
+    force on inputs with planted exact ties: where the argmin ties with a bit-identical copy, the
+    oracle must report P2 == P (a tie is not a strict gap) and the lowest tied index (G2);
+    elsewhere P2 equals the brute-force second-best value."""
+    d, n, m = 3, 70, 8
+    if ab:
+        Tq, Tr = datagen.random_walk_ab(d, n, m, 41, motif=False)
+        Tr = _plant_copies(Tr, m, 10, [30, 55])
+        P, I, P2 = oracle_mod.mstamp(Tq, m, Tr=Tr)
+        Pb, Ib, P2b = brute.mstamp(Tq, m, 0, Tr=Tr)
+    else:
+        Tq, Tr = _plant_copies(datagen.random_walk(d, n, m, 41, motif=False), m, 5, [30, 52]), None
+        P, I, P2 = oracle_mod.mstamp(Tq, m, 2)
+        Pb, Ib, P2b = brute.mstamp(Tq, m, 2)
+    tol = _near_tol(Pb, m, rtol=1e-11) + 1e-13
+    assert np.all(np.abs(P - Pb) <= tol)
+    assert np.all(np.abs(P2 - P2b) <= _near_tol(P2b, m, rtol=1e-11) + 1e-13)
+    copies = {10, 30, 55} if ab else {5, 30, 52}
+    tied = np.isin(I, list(copies))
+    assert tied.sum() > 0
+    # an exact tie between bit-identical windows: runner-up equals the best, index is the lowest copy
+    for k, i in zip(*np.nonzero(tied)):
+        others = [j for j in copies if j != I[k, i] and (ab or abs(j - i) > 2)]
+        if others:
+            assert P2[k, i] == P[k, i], (k, i)
+            assert I[k, i] == min([I[k, i]] + others), (k, i)
+    # away from ties, the strict gap is positive and the index agrees with the brute force
+    _check_index(P, I, P2, Ib, Pb, 1e-9)
+    assert np.mean((P2 - P) > 1e-9) > 0.5
 
 
 def test_cell_matches_direct_definition(oracle_mod):
@@ -199,6 +246,22 @@ def test_flat_window_convention(oracle_mod):
     T[0, 40:40 + m] = 5.0
     out = oracle_mod.cell(T, m, 40, 80)
     assert out[0] == math.sqrt(2 * m)
+
+
+def test_flat_windows_vs_bruteforce(oracle_mod):
+    """Whole profiles with flat runs (several flat windows in a row, flat against flat, flat in one
+    dimension only) against the brute force with G4 applied explicitly."""
+    d, n, m, e = 2, 120, 8, 2
+    T = datagen.random_walk(d, n, m, 42, motif=False)
+    T[0, 20:40] = 1.5      # 13 consecutive flat windows in dim 0
+    T[0, 80:90] = -2.0     # 3 more, far away (flat vs flat cells)
+    T[1, 60:70] = 0.25
+    P, I, P2 = oracle_mod.mstamp(T, m, e)
+    Pb, Ib, P2b = brute.mstamp(T, m, e)
+    assert np.all(np.abs(P - Pb) <= _near_tol(Pb, m, rtol=1e-11) + 1e-13)
+    assert np.all(np.abs(P2 - P2b) <= _near_tol(P2b, m, rtol=1e-11) + 1e-13)
+    _check_index(P, I, P2, Ib, Pb, 1e-9)
+    assert np.allclose(brute.dist_cube(T, m)[0, 21, 81], math.sqrt(2 * m))
 
 
 def test_sampled_rows_equal_full(oracle_mod, c1):
