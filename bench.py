@@ -1,10 +1,13 @@
 """Benchmark of the mSTAMP hot path (BASELINE.json metric: d*n^2 matrix-profile cells*dims/s).
 
 A "step" = one whole pass of the hot path (precompute -> fused diagonal kernel ->
-finalize) over the workload, inputs resident in HBM.  Default workload: BASELINE
-config C2 (self-join, d=16, n=65536, m=128, seeded random walk + planted motif), the
-configuration the metric is quoted on, FP32 headline; every precision is also timed
-and reported under "per_precision".
+finalize) over the workload, inputs resident in HBM.  BASELINE.json's metric names no
+configuration, so the headline runs the largest single-GPU config, C3 (self-join, d=64,
+n=262144, m=256, seeded random walk + planted motif), in FP32; Mixed, FP16 and FP64 are timed
+on the same workload under "per_precision", C2 (d=16) is reported as context, and one
+diagonal band of C4 / C5 at full input size under "per_config_band".  With --gpus N > 1 the
+default workload is C4 (AB-join d=128, n=2^20, m=256), the config BASELINE names for
+1/2/4/8 GPUs.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--precision fp32] [--config C2]
   python bench.py --impl reference ...   (the FP64 CPU oracle on host cores, sampled rows)
@@ -76,9 +79,20 @@ def batcher_ce(N: int) -> int:
 
 
 def alu_ops_per_cell_dim(d: int, self_join: bool) -> float:
-    """Algorithmic ALU-pipe ops per computed cell*dim: the d-way sort
-    network (2 FMNMX per comparator, padded to a power of two) + 1 threshold compare per
-    profile side updated (row; + column for the self-join)."""
+    """Algorithmic ALU-pipe ops per computed cell*dim: clamp 1 + the d-way sort
+    network (2 min/max per Batcher comparator, padded to a power of two, per dim) + the
+    min-update, 3 per profile side (row; + column for the self-join): 9.5 / 14.9 / 24 / 27 / 37
+    for C1..C5.  This is the roofline's op count."""
+    dp = 1
+    while dp < d:
+        dp <<= 1
+    return 1.0 + 2.0 * batcher_ce(dp) / d + 3.0 * (2.0 if self_join else 1.0)
+
+
+def alu_ops_filtered(d: int, self_join: bool) -> float:
+    """The same count for the filtered design the kernels implement (no clamp: |.| is a free
+    operand modifier; one threshold compare per side instead of the 3-op min-update; the
+    update itself runs on the rare cells that pass): a second, stricter figure."""
     dp = 1
     while dp < d:
         dp <<= 1
@@ -220,27 +234,41 @@ def launches_per_step(prec: str, self_join: bool) -> int:
 # ---------------------------------------------------------------------------- CPU oracle leg
 def oracle_sample(cfg, target_s: float = 15.0, max_rows: int = 8192):
     """Time the FP64 oracle (as it stands) on sampled query rows of the workload.
-    Returns (cell*dims per second, rows, seconds, threads)."""
+    Returns (cell*dims per second, rows, seconds, threads, how).  Each sampled row is one query
+    window against all n reference windows x d dims.  Small configs run oracle.mstamp (window
+    statistics of the whole series once, then the rows); where those statistics alone would take
+    longer than the sample (n d m > 2e9, C3..C5) the rows run oracle.mstamp_band over every
+    diagonal, which computes each window's statistics where it needs them."""
     import oracle
     oracle.build()
     T, Tr, m, e, n, d = cfg["T"], cfg["Tr"], cfg["m"], cfg["exclusion"], cfg["n"], cfg["d"]
     threads = os.cpu_count() or 1
     rng = np.random.default_rng(0)
+    big = n * d * m > 2e9
+    how = "oracle.mstamp_band (all diagonals)" if big else "oracle.mstamp"
+
+    def run(rows):
+        if big:
+            lo, hi = (0, n) if Tr is None else (-(n - 1), n)
+            oracle.mstamp_band(T, m, rows, lo, hi, e, Tr=Tr, nthreads=threads)
+        else:
+            oracle.mstamp(T, m, e, Tr=Tr, rows=rows, nthreads=threads)
+
     rows = np.sort(rng.choice(n, size=min(threads, n), replace=False))
     t0 = time.perf_counter()
-    oracle.mstamp(T, m, e, Tr=Tr, rows=rows, nthreads=threads)
+    run(rows)
     dt = time.perf_counter() - t0
     for _ in range(2):  # calibrate (the first call also pays the O(n d m) window stats)
         nr = int(min(max_rows, max(len(rows), len(rows) * target_s / max(dt, 1e-6))))
         nr = max(threads, (nr // threads) * threads)
         rows = np.sort(rng.choice(n, size=min(nr, n), replace=False))
         t0 = time.perf_counter()
-        oracle.mstamp(T, m, e, Tr=Tr, rows=rows, nthreads=threads)
+        run(rows)
         dt = time.perf_counter() - t0
         if dt > 0.5 * target_s or nr >= max_rows:
             break
     cells = len(rows) * n * d          # each sampled row: all n reference windows x d dims
-    return cells / dt, len(rows), dt, threads
+    return cells / dt, len(rows), dt, threads, how
 
 
 def run_reference(args):
@@ -253,16 +281,17 @@ def run_reference(args):
         oracle_sample(cfg, target_s=2.0)
     meta = None
     for _ in range(args.steps):
-        v, nr, dt, th = oracle_sample(cfg, target_s=args.ref_seconds)
+        v, nr, dt, th, how = oracle_sample(cfg, target_s=args.ref_seconds)
         vals.append(v)
-        meta = (nr, dt, th)
+        meta = (nr, dt, th, how)
     value = statistics.mean(vals)
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": meta[1] * 1e3,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic", "config": config_json(args, cfg),
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": meta[2], "kind": "oracle",
-                             "sample": f"{meta[0]} random query rows x all n reference windows per step"},
+                             "precision": "fp64",
+                             "sample": f"{meta[0]} random query rows x all n reference windows per step ({meta[3]})"},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -278,33 +307,63 @@ def config_json(args, cfg):
 
 
 # ---------------------------------------------------------------------------- GPU leg
+def property_check(P, I, cfg):
+    """Oracle-free checks of a (merged) profile at every (k, i): the distance bound
+    0 <= P <= 2 sqrt(m), P non-decreasing in k, finite where an admissible j exists, and the
+    planted motif found in its dimensions (I[k][a] = b).  Used for the multi-GPU merge, whose
+    full 1-GPU recomputation would take minutes to hours at C4 / C5."""
+    import torch
+    m, d, n = cfg["m"], cfg["d"], cfg["n"]
+    fin = torch.isfinite(P)
+    ok_bound = bool(((P[fin] >= 0) & (P[fin] <= 2 * math.sqrt(m) * (1 + 1e-6))).all())
+    diff = torch.diff(torch.where(fin, P, torch.zeros_like(P)), dim=0)
+    ok_mono = bool((diff >= -1e-6 * torch.where(fin[1:], P[1:], torch.ones_like(P[1:]))).all())
+    ok_idx = bool(((I[fin] >= 0) & (I[fin] < n)).all())
+    pos = datagen.motif_positions(n, m)
+    ok_motif = None
+    if pos is not None:
+        a, b = pos
+        ok_motif = bool((I[: max(1, d // 2), a] == b).all())
+    return {"bound": ok_bound, "monotone_in_k": ok_mono, "index_range": ok_idx, "planted_motif": ok_motif}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--precision", default="fp32")
-    ap.add_argument("--config", default="C2")
+    ap.add_argument("--config", default=None, help="C1..C5 (default: C3 at N = 1, C4 at N > 1)")
     ap.add_argument("--impl", default="native", choices=["native", "reference"])
     ap.add_argument("--ref-seconds", type=float, default=15.0)
     ap.add_argument("--no-per-precision", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-context", action="store_true", help="skip the C2 context line")
     ap.add_argument("--no-per-config", action="store_true",
                     help="skip the one-band throughput probes of the larger BASELINE configs")
+    ap.add_argument("--merge-check", default="auto", choices=["auto", "full", "properties", "off"],
+                    help="N > 1: 'full' recomputes the job on one GPU and compares bit for bit (C1/C2: "
+                         "'auto'), 'properties' checks bound / monotonicity / planted motif (larger configs)")
     ap.add_argument("--backend", default="nccl", help="process-group backend for N>1 (gloo: functional "
                     "test of the multi-rank path, e.g. several ranks on one GPU via MP_BENCH_DEVICE)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if args.config is None:
+        args.config = "C3" if world == 1 else "C4"
     if args.impl == "reference":
         return run_reference(args)
 
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("MP_BENCH_DEVICE", os.environ.get("LOCAL_RANK", "0")))
+    if world > 1 and args.backend == "nccl":
+        # NCCL init logging: the communicator's size and transport (NVLink / NVLS) go to stderr
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
     import torch
     import torch.distributed as dist
     from paper_conf_ipps_juryl022_b200 import mstamp
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("MP_BENCH_DEVICE", os.environ.get("LOCAL_RANK", "0")))
     torch.cuda.set_device(local)
     if world > 1:
         if args.backend == "nccl":
@@ -312,91 +371,133 @@ def main():
         else:
             dist.init_process_group(args.backend)
     dev = torch.device("cuda", local)
-    cfg = datagen.make(args.config)
-    d, n, m, e = cfg["d"], cfg["n"], cfg["m"], cfg["exclusion"]
-    self_join = cfg["Tr"] is None
-    T = torch.from_numpy(cfg["T"]).to(dev)
-    Tr = None if self_join else torch.from_numpy(cfg["Tr"]).to(dev)
     ctx = mstamp.Context(local)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream(dev)
 
-    last = {}
+    def load_cfg(name):
+        cfg = datagen.make(name)
+        T = torch.from_numpy(cfg["T"]).to(dev)
+        Tr = None if cfg["Tr"] is None else torch.from_numpy(cfg["Tr"]).to(dev)
+        return cfg, T, Tr
 
-    def one_step(prec):
-        """One pass of the whole hot path; returns (device ms, main-kernel ms)."""
+    def runner(cfg, T, Tr):
+        d, n, m, e = cfg["d"], cfg["n"], cfg["m"], cfg["exclusion"]
         P = torch.empty(d, n, dtype=torch.float64, device=dev)
         I = torch.empty(d, n, dtype=torch.int64, device=dev)
-        last["P"], last["I"], last["prec"] = P, I, prec
-        flush.fill_(1)
-        if world > 1:
-            dist.barrier()
-        torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        if world == 1:
-            ctx.compute_device(T, m, P, I, prec, e, Tr=Tr, stream=stream)
-        else:
-            keys = torch.empty(mstamp.key_words(d, n, prec), dtype=torch.int64, device=dev)
-            ctx.partial_device(T, m, keys, rank, world, prec, e, Tr=Tr, stream=stream)
-            mstamp.merge_partials(ctx, keys, d, n, prec)
-            if rank == 0:
-                ctx.finalize_device(d, n, keys, P, I, prec, stream=stream)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        kms, _ = ctx.last_timing()
-        return e0.elapsed_time(e1), kms
+        keys = {}
 
-    def timed(prec, steps, warm, sample_clocks=False):
-        for _ in range(warm):
-            one_step(prec)
-        cs = ClockSampler(local) if sample_clocks else None
-        if cs:
-            cs.start()
-            time.sleep(0.3)
-        ms, kms = [], []
-        for _ in range(steps):
-            a, b = one_step(prec)
-            ms.append(a)
-            kms.append(b)
-        clocks = cs.stop() if cs else None
-        tot = torch.tensor([sum(ms)], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(tot, op=dist.ReduceOp.MAX)
-        return tot.item() / steps, statistics.mean(kms), clocks
+        def one_step(prec):
+            """One pass of the whole hot path; returns (device ms, main-kernel ms)."""
+            flush.fill_(1)
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            if world == 1:
+                ctx.compute_device(T, m, P, I, prec, e, Tr=Tr, stream=stream)
+            else:
+                if prec not in keys:
+                    keys[prec] = torch.empty(mstamp.key_words(d, n, prec), dtype=torch.int64, device=dev)
+                k = keys[prec]
+                ctx.partial_device(T, m, k, rank, world, prec, e, Tr=Tr, stream=stream)
+                mstamp.merge_partials(ctx, k, d, n, prec)
+                if rank == 0:
+                    ctx.finalize_device(d, n, k, P, I, prec, stream=stream)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            kms, _ = ctx.last_timing()
+            return e0.elapsed_time(e1), kms
 
+        def timed(prec, steps, warm, sample_clocks=False):
+            for _ in range(warm):
+                one_step(prec)
+            cs = ClockSampler(local) if sample_clocks else None
+            if cs:
+                cs.start()
+                time.sleep(0.3)
+            ms, kms = [], []
+            for _ in range(steps):
+                a, b = one_step(prec)
+                ms.append(a)
+                kms.append(b)
+            clocks = cs.stop() if cs else None
+            tot = torch.tensor([sum(ms)], dtype=torch.float64, device=dev)
+            if world > 1:
+                dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+            return tot.item() / steps, statistics.mean(kms), clocks
+
+        return timed, P, I
+
+    cfg, T, Tr = load_cfg(args.config)
+    d, n, m, e = cfg["d"], cfg["n"], cfg["m"], cfg["exclusion"]
+    self_join = cfg["Tr"] is None
+    timed, Plast, Ilast = runner(cfg, T, Tr)
     ms, kms, clocks = timed(args.precision, args.steps, args.warmup, sample_clocks=True)
-    merge_check = None
-    if world > 1 and rank == 0:
-        # outside the timed region: the merged N-rank result must equal the 1-GPU result bit
-        # for bit (fixed tile plan, lexicographic MINLOC merge: DESIGN.md section 10)
-        P1 = torch.empty(d, n, dtype=torch.float64, device=dev)
-        I1 = torch.empty(d, n, dtype=torch.int64, device=dev)
-        ctx.compute_device(T, m, P1, I1, args.precision, e, Tr=Tr, stream=stream)
-        torch.cuda.synchronize()
-        merge_check = {"bit_identical_to_1gpu": bool(torch.equal(P1, last["P"]) and torch.equal(I1, last["I"]))}
-        del P1, I1
+    run_mhz = (clocks or {}).get("sm_mhz") or NOMINAL_SM_MHZ
     dn2 = d * n * n
     value = dn2 / (ms * 1e-3)
 
+    merge_check = None
+    if world > 1:
+        mode = args.merge_check
+        if mode == "auto":
+            mode = "full" if args.config in ("C1", "C2") else "properties"
+        if rank == 0 and mode == "full":
+            # outside the timed region: the merged N-rank result must equal the 1-GPU result bit
+            # for bit (fixed tile plan, lexicographic MINLOC merge: DESIGN.md section 10)
+            P1 = torch.empty(d, n, dtype=torch.float64, device=dev)
+            I1 = torch.empty(d, n, dtype=torch.int64, device=dev)
+            ctx.compute_device(T, m, P1, I1, args.precision, e, Tr=Tr, stream=stream)
+            torch.cuda.synchronize()
+            merge_check = {"bit_identical_to_1gpu": bool(torch.equal(P1, Plast) and torch.equal(I1, Ilast))}
+            del P1, I1
+        elif rank == 0 and mode == "properties":
+            merge_check = property_check(Plast, Ilast, cfg)
+
+    cells = computed_cells(n, e, self_join)
+    peak_ops = alu_peak_ops(run_mhz)
+
+    def frac(kms_, d_, cells_, self_, prec_):
+        rate = cells_ * d_ / (kms_ * 1e-3)
+        return rate * alu_ops_mode(d_, self_, prec_) / peak_ops
+
     per_prec = {}
     if not args.no_per_precision:
-        for prec in ("fp64", "fp32", "mixed", "fp16"):
+        for prec in ("fp32", "mixed", "fp16", "fp64"):
             if prec == args.precision:
-                per_prec[prec] = {"value": value, "ms_per_step": ms, "main_kernel_ms": kms}
-                continue
-            p_ms, p_kms, _ = timed(prec, max(1, min(args.steps, 3)), 1)
-            per_prec[prec] = {"value": dn2 / (p_ms * 1e-3), "ms_per_step": p_ms, "main_kernel_ms": p_kms}
-        cells0 = computed_cells(n, e, self_join)
-        for prec, v in per_prec.items():  # ALU roofline fraction of the main kernel per mode
-            rate = cells0 * d / (v["main_kernel_ms"] * 1e-3)
-            v["alu_frac"] = rate * alu_ops_mode(d, self_join, prec) / alu_peak_ops((clocks or {}).get("sm_mhz"))
+                per_prec[prec] = {"value": value, "ms_per_step": ms, "main_kernel_ms": kms, "steps": args.steps}
+            else:
+                # FP64 takes ~50 s per C3 step: one warm-up, one timed step
+                st, wu = (1, 1) if prec == "fp64" and d * n * n > 1e12 else (max(1, min(args.steps, 3)), 1)
+                p_ms, p_kms, _ = timed(prec, st, wu)
+                per_prec[prec] = {"value": dn2 / (p_ms * 1e-3), "ms_per_step": p_ms, "main_kernel_ms": p_kms,
+                                  "steps": st}
+            per_prec[prec]["alu_frac"] = frac(per_prec[prec]["main_kernel_ms"], d, cells, self_join, prec)
+            per_prec[prec]["computed_cell_dims_per_s"] = cells * d / (per_prec[prec]["main_kernel_ms"] * 1e-3)
+
+    context = None
+    if not args.no_context and world == 1 and args.config != "C2":
+        c2, T2, Tr2 = load_cfg("C2")
+        timed2, _, _ = runner(c2, T2, Tr2)
+        context = {"workload": "C2: self-join d=16 n=65536 m=128", "per_precision": {}}
+        cells2 = computed_cells(c2["n"], c2["exclusion"], True)
+        for prec in ("fp32", "mixed", "fp16", "fp64"):
+            p_ms, p_kms, _ = timed2(prec, 3, 1)
+            context["per_precision"][prec] = {
+                "value": c2["d"] * c2["n"] ** 2 / (p_ms * 1e-3), "ms_per_step": p_ms, "main_kernel_ms": p_kms,
+                "alu_frac": frac(p_kms, c2["d"], cells2, True, prec)}
+        del T2, Tr2, timed2
+        torch.cuda.empty_cache()
 
     per_cfg = {}
     if not args.no_per_config and world == 1:
-        for name, prec in (("C3", "fp32"), ("C3", "mixed"), ("C3", "fp16"), ("C4", "fp32"), ("C4", "mixed"),
-                           ("C4", "fp64"), ("C5", "fp32"), ("C5", "mixed"), ("C5", "fp16"), ("C5", "fp64")):
-            per_cfg[f"{name}/{prec}"] = band_probe(ctx, torch, dev, name, prec, peak=alu_peak_ops((clocks or {}).get("sm_mhz")))
+        for name, prec in (("C4", "fp32"), ("C4", "mixed"), ("C4", "fp64"), ("C5", "fp32"), ("C5", "mixed"),
+                           ("C5", "fp16"), ("C5", "fp64")):
+            if name == args.config:
+                continue
+            per_cfg[f"{name}/{prec}"] = band_probe(ctx, torch, dev, name, prec, peak=peak_ops)
         _PROBE_CACHE.clear()
         torch.cuda.empty_cache()
 
@@ -423,38 +524,41 @@ def main():
 
     if rank == 0:
         peaks, src = load_peaks()
-        cells = computed_cells(n, e, self_join)
         # roofline of the dominant kernel: algorithmic ops of the cells THIS launch computed (rank
         # 0's band when N > 1) over its CUDA-event duration
         band_cells = cells
         if world > 1:
             _, bc = mstamp.plan_bands(d, n, m, args.precision, e, self_join, world)
             band_cells = int(bc[0])
-        ops = alu_ops_per_cell_dim(d, self_join) * band_cells * d
+        ops = alu_ops_mode(d, self_join, args.precision) * band_cells * d
         lanes, lsrc = alu_lanes()
-        run_mhz = (clocks or {}).get("sm_mhz") or NOMINAL_SM_MHZ
-        peak_tops = alu_peak_ops(run_mhz) / 1e12
+        peak_tops = peak_ops / 1e12
         achieved = ops / (kms * 1e-3) / 1e12 if kms > 0 else None
+        kname = {"fp32": "mp_diag_cta" if d > 32 else "mp_diag", "fp64": "mp_diag_cta64" if d > 32 else "mp_diag64f"}
         roof = {"bound": "alu", "achieved": achieved, "peak": peak_tops, "unit": "Tops/s",
                 "frac": achieved / peak_tops if achieved else None,
                 "traffic": load_traffic(args.config, args.precision),
-                "kernel": "mp_diag", "ops_per_cell_dim": alu_ops_per_cell_dim(d, self_join),
+                "kernel": kname.get(args.precision, "mp_diag_cta_h" if d > 32 else "mp_diag_h"),
+                "ops_per_cell_dim": alu_ops_mode(d, self_join, args.precision),
+                "ops_basis": "SURVEY 8(d): clamp 1 + 2 CE(d_pad)/d + 3 per profile side",
+                "frac_filtered_ops": (alu_ops_filtered(d, self_join) * band_cells * d / (kms * 1e-3) / 1e12 / peak_tops
+                                      / (2.0 if args.precision in ("fp16", "mixed", "fp16c") else 1.0)) if kms > 0 else None,
                 "computed_cell_dims": band_cells * d,
                 "peak_basis": f"{SM_COUNT} SM x {lanes:.2f} FMNMX lanes/SM/clk ({lsrc}: scripts/pipe_peaks.cu -> "
                               f"profiles/r1_pipe_peaks.json; MEASURED_PEAKS {src} has no ALU figure) x {run_mhz:.0f} MHz "
                               "(SM clock sampled during the timed region)"}
         cpu = None
         if not args.no_cpu_baseline and world == 1:
-            v, nr, dt, th = oracle_sample(cfg, target_s=args.ref_seconds)
-            cpu = {"value": v, "unit": UNIT, "cores": th, "kind": "oracle",
-                   "sample": f"{nr} random query rows x all {n} reference windows ({dt:.1f} s)"}
+            v, nr, dt, th, how = oracle_sample(cfg, target_s=args.ref_seconds)
+            cpu = {"value": v, "unit": UNIT, "cores": th, "kind": "oracle", "precision": "fp64",
+                   "sample": f"{nr} random query rows x all {n} reference windows ({dt:.1f} s, {how})"}
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
                 "vs_baseline": None, "dtype": {"fp64": "f64", "fp32": "f32"}.get(args.precision, args.precision),
                 "data": "synthetic", "config": config_json(args, cfg), "roofline": roof, "cpu_baseline": cpu,
                 "e2e": e2e, "gpu_launches": launches_per_step(args.precision, self_join) * args.steps,
-                "clocks": clocks, "per_precision": per_prec, "per_config_band": per_cfg or None,
-                "computed_cells_per_s": cells * d / (ms * 1e-3)}
+                "clocks": clocks, "per_precision": per_prec, "context": context,
+                "per_config_band": per_cfg or None, "computed_cells_per_s": cells * d / (ms * 1e-3)}
         if merge_check is not None:
             line["merge_check"] = merge_check
         print(json.dumps(line), flush=True)

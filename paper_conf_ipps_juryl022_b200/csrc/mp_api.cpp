@@ -48,6 +48,7 @@ struct mp_ctx {
     Buf dT, dTr, st_q, st_r, tw_q, tw_r, mu_q, mu_r, mup_q, mup_r, nrm, keys, ext, seg, counter, dP, dI, flag;
     Buf stp_q, stp_r, scale, maxbits, flat;  // FP16 / Mixed precompute
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    int* hflag = nullptr;   // pinned read-back of the non-finite flag
     double last_ms = 0.0;
     int64_t last_launches = 0;
 };
@@ -177,15 +178,14 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     H = std::min<int64_t>((H + 7) / 8 * 8, int64_t(1) << 30);
     if (self && excl < 0) excl = (m + 3) / 4;
 
-    // flag non-finite inputs (reading G23)
+    // flag non-finite inputs (reading G23).  The flag is read back after the whole pipeline is
+    // enqueued (finish_partial), so the check costs one O(d L) kernel and no mid-pipeline host
+    // sync; a non-finite input only makes the kernels compute NaN distances, which never pass
+    // a profile update, before the call reports MP_ERR_INVALID.
     MP_CUDA(ctx, ensure(ctx->flag, sizeof(int)));
     MP_CUDA(ctx, cudaMemsetAsync(ctx->flag.p, 0, sizeof(int), s));
     MP_CUDA(ctx, mpk::launch_check_finite(dT, d * L, (int*)ctx->flag.p, s));
     if (!self) MP_CUDA(ctx, mpk::launch_check_finite(dTr, d * L, (int*)ctx->flag.p, s));
-    int flag = 0;
-    MP_CUDA(ctx, cudaMemcpyAsync(&flag, ctx->flag.p, sizeof(int), cudaMemcpyDeviceToHost, s));
-    MP_CUDA(ctx, cudaStreamSynchronize(s));
-    if (flag) return fail(ctx, MP_ERR_INVALID, "non-finite input");
 
     // precalculation (Pseudocode 1 line 2)
     const bool half = prec == MP_FP16 || prec == MP_MIXED || prec == MP_FP16C;
@@ -221,7 +221,7 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
 
     // keys (FP16 / Mixed use the FP32 key format: float bits of the half-precision sum)
     const size_t kb = (size_t)n * d * (prec == MP_FP64 ? 16 : 8);
-    MP_CUDA(ctx, ensure(ctx->keys, kb));
+    MP_CUDA(ctx, ensure(ctx->keys, kb + 16));   // + 16: TMA key rows are 16-byte aligned supersets
     MP_CUDA(ctx, mpk::launch_init_keys(prec, ctx->keys.p, n * d, s));
 
     // plan + band
@@ -303,6 +303,16 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     return MP_OK;
 }
 
+// Read back the non-finite flag of the last run_partial (after the caller's remaining work on
+// stream s is enqueued): one pinned 4-byte copy and a stream sync.
+mp_status finish_partial(mp_ctx* ctx, cudaStream_t s) {
+    if (!ctx->hflag) MP_CUDA(ctx, cudaHostAlloc((void**)&ctx->hflag, sizeof(int), cudaHostAllocDefault));
+    MP_CUDA(ctx, cudaMemcpyAsync(ctx->hflag, ctx->flag.p, sizeof(int), cudaMemcpyDeviceToHost, s));
+    MP_CUDA(ctx, cudaStreamSynchronize(s));
+    if (*ctx->hflag) return fail(ctx, MP_ERR_INVALID, "non-finite input");
+    return MP_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -343,6 +353,7 @@ void mp_free(mp_ctx* ctx) {
                    &ctx->mu_r, &ctx->mup_q, &ctx->mup_r, &ctx->nrm, &ctx->keys, &ctx->ext, &ctx->seg, &ctx->counter, &ctx->dP,
                    &ctx->dI, &ctx->flag, &ctx->stp_q, &ctx->stp_r, &ctx->scale, &ctx->maxbits, &ctx->flat};
     for (Buf* b : bufs) release(*b);
+    if (ctx->hflag) cudaFreeHost(ctx->hflag);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
     if (ctx->ev1) cudaEventDestroy(ctx->ev1);
     if (ctx->stream) cudaStreamDestroy(ctx->stream);
@@ -401,7 +412,7 @@ mp_status mp_partial_device(mp_ctx* ctx, void* cuda_stream, const double* dT, co
     st = run_partial(ctx, s, dT, dTr, d, n, m, prec, exclusion, rank, world);
     if (st != MP_OK) return st;
     MP_CUDA(ctx, mpk::launch_keys_to_ext(prec, ctx->keys.p, dKeys, n * d, s));
-    return MP_OK;
+    return finish_partial(ctx, s);
 }
 
 mp_status mp_key_mask_device(mp_ctx* ctx, void* cuda_stream, int64_t d, int64_t n, int64_t* dKeys,
@@ -440,7 +451,7 @@ mp_status mp_compute_device(mp_ctx* ctx, void* cuda_stream, const double* dT, co
     } else {
         MP_CUDA(ctx, mpk::launch_finalize(prec, ctx->keys.p, n, (int)d, dP, (long long*)dI, s));
     }
-    return MP_OK;
+    return finish_partial(ctx, s);
 }
 
 mp_status mp_compute(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, int64_t n, int64_t m,

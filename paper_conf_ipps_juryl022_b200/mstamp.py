@@ -118,6 +118,25 @@ def _tptr(t):
     return None if t is None else ctypes.c_void_p(t.data_ptr())
 
 
+def _need(t, name, dtype, device, shape=None, min_numel=None):
+    """Argument marshalling guard: a torch tensor of the dtype, on the context's device,
+    contiguous and of the shape the C ABI reads or writes (else MPError(MP_ERR_INVALID) before
+    any device pointer crosses the boundary)."""
+    import torch
+    if not isinstance(t, torch.Tensor):
+        raise MPError(1, f"{name} must be a torch tensor")
+    if t.dtype != dtype:
+        raise MPError(1, f"{name} must be {dtype}, got {t.dtype}")
+    if t.device.type != "cuda" or t.device.index != device:
+        raise MPError(1, f"{name} must live on cuda:{device}, got {t.device}")
+    if not t.is_contiguous():
+        raise MPError(1, f"{name} must be contiguous")
+    if shape is not None and tuple(t.shape) != tuple(shape):
+        raise MPError(1, f"{name} must have shape {tuple(shape)}, got {tuple(t.shape)}")
+    if min_numel is not None and t.numel() < min_numel:
+        raise MPError(1, f"{name} needs >= {min_numel} elements, has {t.numel()}")
+
+
 class Context:
     """One context per host thread / GPU (mp_init ... mp_free)."""
 
@@ -186,8 +205,13 @@ class Context:
     # ---- device memory (torch tensors)
     def compute_device(self, T, m, P, I, prec="fp32", exclusion=-1, Tr=None, stream=None):
         import torch
+        _need(T, "T", torch.float64, self.device)
         d, L = T.shape
         n = L - m + 1
+        if Tr is not None:
+            _need(Tr, "Tr", torch.float64, self.device, shape=T.shape)
+        _need(P, "P", torch.float64, self.device, shape=(d, n))
+        _need(I, "I", torch.int64, self.device, shape=(d, n))
         s = stream if stream is not None else torch.cuda.current_stream(T.device)
         st = load().mp_compute_device(self._ctx, ctypes.c_void_p(s.cuda_stream), _tptr(T), _tptr(Tr),
                                       d, n, m, _prec(prec), int(exclusion), _tptr(P), _tptr(I))
@@ -195,8 +219,12 @@ class Context:
 
     def partial_device(self, T, m, keys, rank, world, prec="fp32", exclusion=-1, Tr=None, stream=None):
         import torch
+        _need(T, "T", torch.float64, self.device)
         d, L = T.shape
         n = L - m + 1
+        if Tr is not None:
+            _need(Tr, "Tr", torch.float64, self.device, shape=T.shape)
+        _need(keys, "keys", torch.int64, self.device, min_numel=key_words(d, n, prec))
         s = stream if stream is not None else torch.cuda.current_stream(T.device)
         st = load().mp_partial_device(self._ctx, ctypes.c_void_p(s.cuda_stream), _tptr(T), _tptr(Tr),
                                       d, n, m, _prec(prec), int(exclusion), int(rank), int(world),
@@ -205,6 +233,8 @@ class Context:
 
     def key_mask_device(self, d, n, keys, global_v, stream=None):
         import torch
+        _need(keys, "keys", torch.int64, self.device, min_numel=2 * d * n)
+        _need(global_v, "global_v", torch.int64, self.device, min_numel=d * n)
         s = stream if stream is not None else torch.cuda.current_stream(keys.device)
         st = load().mp_key_mask_device(self._ctx, ctypes.c_void_p(s.cuda_stream), d, n, _tptr(keys),
                                        _tptr(global_v))
@@ -212,6 +242,9 @@ class Context:
 
     def finalize_device(self, d, n, keys, P, I, prec="fp32", stream=None):
         import torch
+        _need(keys, "keys", torch.int64, self.device, min_numel=key_words(d, n, prec))
+        _need(P, "P", torch.float64, self.device, shape=(d, n))
+        _need(I, "I", torch.int64, self.device, shape=(d, n))
         s = stream if stream is not None else torch.cuda.current_stream(keys.device)
         st = load().mp_finalize_device(self._ctx, ctypes.c_void_p(s.cuda_stream), d, n, _prec(prec),
                                        _tptr(keys), _tptr(P), _tptr(I))

@@ -28,12 +28,20 @@ def test_batcher_comparator_counts(N, ce):
         assert ce == (p * p - p + 4) * 2 ** (p - 2) - 1
 
 
-def test_alu_ops_model():
-    # 2 FMNMX per comparator of the padded network / d + 1 compare per side
-    assert bench.alu_ops_per_cell_dim(16, True) == pytest.approx(2 * 63 / 16 + 2)
-    assert bench.alu_ops_per_cell_dim(16, False) == pytest.approx(2 * 63 / 16 + 1)
-    assert bench.alu_ops_per_cell_dim(12, True) == pytest.approx(2 * 63 / 12 + 2)   # padded to 16
+@pytest.mark.parametrize("cfg,ops", [("C1", 9.5), ("C2", 14.9), ("C3", 24), ("C4", 27), ("C5", 37)])
+def test_alu_ops_model_matches_survey(cfg, ops):
+    """The roofline's op count per computed cell*dim reproduces SURVEY.md 8(d)'s table (clamp 1 +
+    2 CE(d_pad)/d + 3 per profile side), written from the paper's algorithm before any kernel:
+    9.5 / 14.9 / 24 / 27 / 37 for C1..C5."""
+    from paper_conf_ipps_juryl022_b200 import datagen
+    join, d, n, m, e, seed = datagen.CONFIGS[cfg]
+    assert bench.alu_ops_per_cell_dim(d, join == "self") == pytest.approx(ops, abs=0.06)
+
+
+def test_alu_ops_half_modes_count_pairs():
+    # half2 instructions serve two cells (DESIGN.md "Roofline")
     assert bench.alu_ops_mode(16, True, "mixed") == pytest.approx(bench.alu_ops_per_cell_dim(16, True) / 2)
+    assert bench.alu_ops_filtered(16, True) < bench.alu_ops_per_cell_dim(16, True)
 
 
 @pytest.mark.parametrize("n,e", [(10, 0), (10, 2), (37, 5), (8, 7), (8, 9)])

@@ -207,6 +207,54 @@ def _half_stats(P_or, I_or, P, I, m):
                 max_rel=float(rel.max()), recall=float((I == I_or)[fin].mean()))
 
 
+# Stated element-wise bounds of the half modes (measured on the full C1 / C2 /
+# C3 grids, profiles/r2_half_bounds.json): |P - P_ref| / sqrt(2m) over every (k, i), maximum and
+# 99.9th percentile.  sqrt(2m) is the distance of two uncorrelated z-normalised windows.
+HALF_BOUND = {"mixed": (0.2, 0.05), "fp16c": (0.2, 0.05), "fp16": (0.5, 0.45)}
+
+
+def _assert_half_bound(P_ref, P, m, prec):
+    fin = np.isfinite(P_ref)
+    assert np.array_equal(fin, np.isfinite(P))
+    e = np.abs(P - P_ref)[fin] / math.sqrt(2 * m)
+    mx, p999 = HALF_BOUND[prec]
+    assert e.max() <= mx and np.quantile(e, 0.999) <= p999, (prec, float(e.max()), float(np.quantile(e, 0.999)))
+    return float(e.max()), float(np.quantile(e, 0.999))
+
+
+@pytest.mark.parametrize("prec", ["mixed", "fp16c", "fp16"])
+@pytest.mark.parametrize("cfg_name", ["C1", "C2", "C3"])
+def test_half_modes_elementwise_bound(ctx, oracle_mod, c1_oracle, cfg_name, prec):
+    """The half modes' stated element-wise error bound (HALF_BOUND) on the BASELINE configs: C1
+    over the full grid against the oracle; C2 and C3 over the full grid against the GPU FP64 path
+    (within 1e-9 of the oracle, test_c1_full / test_c2_sampled_rows / test_fp32_full_grid) and
+    on sampled rows against the oracle itself.  Parity of these modes is unpinned (no paper
+    value to pin to); the bound is measured and stated."""
+    if cfg_name == "C1":
+        cfg, P, I, _ = c1_oracle
+        Pg, Ig = ctx.compute(cfg["T"], cfg["m"], prec, cfg["exclusion"])
+        print(cfg_name, prec, "vs oracle (full grid)", _assert_half_bound(P, Pg, cfg["m"], prec))
+        return
+    cfg = datagen.make(cfg_name)
+    T, m, e, n, d = cfg["T"], cfg["m"], cfg["exclusion"], cfg["n"], cfg["d"]
+    Td = torch.from_numpy(T).cuda()
+    P64 = torch.empty(d, n, dtype=torch.float64, device="cuda")
+    I64 = torch.empty(d, n, dtype=torch.int64, device="cuda")
+    ctx.compute_device(Td, m, P64, I64, "fp64", e)
+    Ph = torch.empty_like(P64)
+    Ih = torch.empty_like(I64)
+    ctx.compute_device(Td, m, Ph, Ih, prec, e)
+    torch.cuda.synchronize()
+    p64, ph = P64.cpu().numpy(), Ph.cpu().numpy()
+    del Td, P64, I64, Ph, Ih
+    print(cfg_name, prec, "vs FP64 (full grid)", _assert_half_bound(p64, ph, m, prec))
+    a, b = datagen.motif_positions(n, m)
+    rows = np.unique(np.concatenate([[0, n - 1, a, b], np.random.default_rng(12).integers(0, n, 12)]))
+    Po, _, _ = oracle_mod.mstamp(T, m, e, rows=rows)
+    e_or = np.abs(ph[:, rows] - Po)[np.isfinite(Po)] / math.sqrt(2 * m)
+    assert e_or.max() <= HALF_BOUND[prec][0], (prec, float(e_or.max()))
+
+
 @pytest.mark.parametrize("prec", ["fp64", "fp32"])
 @pytest.mark.parametrize("shape", [(3, 1500, 1024, 256, 81), (16, 900, 600, 150, 82), (70, 400, 300, 75, 83)])
 def test_long_windows(ctx, oracle_mod, prec, shape):
@@ -221,7 +269,7 @@ def test_long_windows(ctx, oracle_mod, prec, shape):
 
 
 @pytest.mark.parametrize("prec", ["fp16", "mixed", "fp16c"])
-def test_half_modes_ab_d16(ctx, prec):
+def test_half_modes_ab_d16(ctx, oracle_mod, prec):
     """AB-join in the half modes at d = 16 (warp half kernel, pairs starting at column -1):
     error vs the GPU FP64 result (oracle-checked elsewhere) within the stated bound, planted
     motif recovered, band partials merge bit-identically."""
@@ -229,10 +277,11 @@ def test_half_modes_ab_d16(ctx, prec):
     d, n, m = 16, 2000, 64
     Tq, Tr = datagen.random_walk_ab(d, n, m, 84)
     Pg, Ig = ctx.compute(Tq, m, prec, Tr=Tr)
-    P64, I64 = ctx.compute(Tq, m, "fp64", Tr=Tr)
-    st = _half_stats(P64, I64, Pg, Ig, m)
+    Po, Io, _ = oracle_mod.mstamp(Tq, m, Tr=Tr)
+    st = _half_stats(Po, Io, Pg, Ig, m)
     print(prec, "ab d16", st)
     assert st["median_rel"] < (0.02 if prec != "fp16" else 0.2)
+    _assert_half_bound(Po, Pg, m, prec)
     a, b = datagen.motif_positions(n, m)
     for k in range(d // 2):
         assert abs(int(Ig[k, a]) - b) <= (0 if prec == "mixed" else m // 16)
@@ -280,8 +329,8 @@ def test_half_modes_c1(ctx, oracle_mod, c1_oracle, prec):
     print(prec, st)
     # stated bounds: Mixed median 2 %, p99 20 %; FP16 (half-precision precalc of an
     # offset random walk, the paper's least accurate mode) median 20 %, p99 100 %
-    med, p99 = (0.02, 0.2) if prec == "mixed" else (0.2, 1.0)
-    assert st["median_rel"] < med and st["p99_rel"] < p99
+    assert st["median_rel"] < (0.02 if prec == "mixed" else 0.2)
+    _assert_half_bound(P, Pg, m, prec)
     assert np.all(Pg >= 0) and np.all(Pg <= 2 * math.sqrt(m) * 1.01)
     a, b = datagen.motif_positions(cfg["n"], m)
     for k in range(max(1, cfg["d"] // 2)):
@@ -299,10 +348,11 @@ def test_half_modes_shapes(ctx, oracle_mod, prec, shape):
     print(prec, shape, st)
     assert st["median_rel"] < (0.05 if prec == "mixed" else 0.2)
     assert np.all(np.isfinite(Pg))
+    print(prec, shape, "element-wise", _assert_half_bound(P, Pg, m, prec))
 
 
 @pytest.mark.parametrize("prec", ["fp16", "mixed", "fp16c"])
-def test_half_modes_ab_and_bands(ctx, prec):
+def test_half_modes_ab_and_bands(ctx, oracle_mod, prec):
     """AB-join runs; band partials merge bit-identically to the single band (FP32 key format)."""
     from paper_conf_ipps_juryl022_b200 import mstamp
     d, n, m = 4, 1500, 32
@@ -311,10 +361,11 @@ def test_half_modes_ab_and_bands(ctx, prec):
     assert np.all(np.isfinite(Pg)) and np.all((Ig >= 0) & (Ig < n))
     # error vs the GPU FP64 result (itself oracle-checked) stays within the stated bound; an
     # AB-join exercises the diagonal starts at column 0 (pairs beginning at column -1)
-    P64, I64 = ctx.compute(Tq, m, "fp64", Tr=Tr)
-    st = _half_stats(P64, I64, Pg, Ig, m)
+    Po, Io, _ = oracle_mod.mstamp(Tq, m, Tr=Tr)
+    st = _half_stats(Po, Io, Pg, Ig, m)
     print(prec, "ab", st)
     assert st["median_rel"] < (0.02 if prec == "mixed" else 0.2)
+    _assert_half_bound(Po, Pg, m, prec)
     a, b = datagen.motif_positions(n, m)
     for k in range(d // 2):
         assert Ig[k, a] == b
@@ -349,6 +400,7 @@ def test_half_modes_large_d(ctx, oracle_mod, prec, shape):
     print(prec, shape, st)
     assert st["median_rel"] < (0.05 if prec == "mixed" else 0.2)
     assert np.all(np.isfinite(Pg)) and np.all((Ig >= 0) & (Ig < n))
+    print(prec, shape, "element-wise", _assert_half_bound(P, Pg, m, prec))
     assert np.all(Pg >= 0) and np.all(Pg <= 2 * math.sqrt(m) * 1.01)
     Td = torch.from_numpy(T).cuda()
     Trd = None if Tr is None else torch.from_numpy(Tr).cuda()
@@ -445,3 +497,64 @@ def test_full_size_band_sampled_rows(ctx, oracle_mod, cfg_name, prec, world):
     assert np.all(Pg[fin] >= 0) and np.all(Pg[fin] <= 2 * math.sqrt(m) * 1.01)
     with np.errstate(invalid="ignore"):
         assert np.all(np.nan_to_num(np.diff(Pg, axis=0), nan=0.0, posinf=0.0) >= -1e-3 * np.nan_to_num(Pg[1:], posinf=0.0))
+
+
+# ---------------------------------------------------------------- FP32 over the full grid (reading R4)
+@pytest.mark.parametrize("shape", ["C3", "X256_32768_512"])
+def test_fp32_full_grid(ctx, oracle_mod, shape):
+    """FP32 at m >= 256 over EVERY (k, i) of the full grid: within tests/parity.py's FP32
+    tolerance of the GPU FP64 path (itself within 1e-9 of the oracle), then the 40 rows worst in
+    units of the tolerance plus the planted motif's neighbourhoods a +- 1..30, b +- 1..30 (where
+    the recurrence error is amplified most) against the oracle itself.  The
+    compensated recurrence (reading R4) is what makes this hold (round 1: C3 26 entries
+    above the tolerance, the d = 256 / m = 512 shape 486)."""
+    if shape == "C3":
+        cfg = datagen.make("C3")
+    else:
+        d_, n_, m_ = (int(v) for v in shape[1:].split("_"))
+        cfg = dict(T=datagen.random_walk(d_, n_, m_, 7), Tr=None, d=d_, n=n_, m=m_, exclusion=m_ // 4)
+    T, m, e, n = cfg["T"], cfg["m"], cfg["exclusion"], cfg["n"]
+    Td = torch.from_numpy(T).cuda()
+    d = cfg["d"]
+    P64 = torch.empty(d, n, dtype=torch.float64, device="cuda")
+    I64 = torch.empty(d, n, dtype=torch.int64, device="cuda")
+    ctx.compute_device(Td, m, P64, I64, "fp64", e)
+    P32 = torch.empty_like(P64)
+    I32 = torch.empty_like(I64)
+    ctx.compute_device(Td, m, P32, I32, "fp32", e)
+    torch.cuda.synchronize()
+    p64, p32, i32 = P64.cpu().numpy(), P32.cpu().numpy(), I32.cpu().numpy()
+    del Td, P64, I64, P32, I32
+    fin = np.isfinite(p64)
+    assert np.array_equal(fin, np.isfinite(p32))
+    tol = parity.tol_of(np.where(fin, p64, 0.0), m, "fp32", P0_row=np.where(fin[0], p64[0], np.inf))
+    r = np.where(fin, np.abs(p32 - p64), 0.0) / np.where(tol > 0, tol, 1.0)
+    print(shape, "full grid err/tol max", float(r.max()), "entries > 1:", int((r > 1).sum()))
+    assert int((r > 1).sum()) == 0, f"{int((r > 1).sum())} entries above the FP32 tolerance (max {r.max():.3f}x)"
+    worst = np.argsort(r.max(axis=0))[::-1][:40]
+    a, b = datagen.motif_positions(n, m)
+    near = [x + o for x in (a, b) for o in range(-30, 31) if o != 0 and 0 <= x + o < n]
+    rows = np.unique(np.concatenate([worst, near]))
+    P, I, P2 = oracle_mod.mstamp(T, m, e, rows=rows)
+    st = parity.check(oracle_mod, T, m, P, I, P2, p32, i32, "fp32", rows=rows)
+    print(shape, "oracle rows", len(rows), st)
+
+
+def test_binding_rejects_bad_tensors(ctx):
+    """The binding checks dtype, device, contiguity and shape before a device pointer crosses the
+    C ABI (a float32 or short output tensor would otherwise be read / written out of bounds)."""
+    from paper_conf_ipps_juryl022_b200 import mstamp
+    d, n, m = 3, 200, 16
+    T = torch.from_numpy(datagen.random_walk(d, n, m, 72)).cuda()
+    P = torch.empty(d, n, dtype=torch.float64, device="cuda")
+    I = torch.empty(d, n, dtype=torch.int64, device="cuda")
+    ctx.compute_device(T, m, P, I, "fp32", 4)
+    for bad in (dict(T=T.float()), dict(P=P[:, :-1]), dict(I=I.int()), dict(P=P.t().contiguous().t()),
+                dict(T=T.cpu())):
+        args = dict(T=T, P=P, I=I)
+        args.update(bad)
+        with pytest.raises(mstamp.MPError):
+            ctx.compute_device(args["T"], m, args["P"], args["I"], "fp32", 4)
+    short = torch.empty(mstamp.key_words(d, n, "fp32") - 1, dtype=torch.int64, device="cuda")
+    with pytest.raises(mstamp.MPError):
+        ctx.partial_device(T, m, short, 0, 1, "fp32", 4)
