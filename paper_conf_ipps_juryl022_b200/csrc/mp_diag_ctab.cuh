@@ -32,13 +32,20 @@
 #define MP_CTAB_NT 128      // threads per block
 #endif
 #ifndef MP_CTAB_MINB16
-#define MP_CTAB_MINB16 3    // resident blocks per SM the register budget is sized for (DL = 16)
+#define MP_CTAB_MINB16 4    // resident blocks per SM the register budget is sized for (DL = 16: 127 registers, no spills)
 #endif
 #ifndef MP_CTAB_MINB32
-#define MP_CTAB_MINB32 2    // ... (DL = 32)
+#define MP_CTAB_MINB32 3    // ... (DL = 32)
 #endif
 #ifndef MP_CTAB_SB
 #define MP_CTAB_SB 0        // steps per staging batch; 0: per G below
+#endif
+#ifndef MP_CTAB_PAIR
+#define MP_CTAB_PAIR 1      // G == 2: the pair-mode merge (pair_si)
+#endif
+#ifndef MP_CTAB_TA
+#define MP_CTAB_TA 1        // thresholds in rank-contiguous per-slot arrays (read as vectors after
+                            // the scan) instead of the stats' 4th word (kept live through the sort)
 #endif
 // dims per lane by padded d (G = d_pad / DL lanes per cell, G <= 32)
 #ifndef MP_CTAB_DL64
@@ -101,13 +108,31 @@ template <int DL, int G, int NT> struct CtabGeo {
     static constexpr int RC = 2 * SB + NCC - 1;
     static constexpr int SS = D + G;                   // V4 slot stride: consecutive slots shift banks
     static constexpr int NTHR = (2 * SB * D + NT - 1) / NT;  // threshold words a thread patches per batch
-    static constexpr size_t ring_bytes = (size_t)(RR + RC) * SS * 16;
+    static constexpr size_t stat_ring_bytes = (size_t)(RR + RC) * SS * 16;
+    static constexpr size_t ring_bytes = stat_ring_bytes + (MP_CTAB_TA ? (size_t)(RR + RC) * D * 4 : 0);
     static constexpr size_t bytes = ring_bytes + 16 /* mbarrier */ + 16 /* tile index */;
 };
 
 // plane (dimension slot) that holds rank r's threshold: lane g holds ranks [g DL, (g+1) DL) at
 // registers kk after the merge and reads plane kk G + g at register kk (rank_of_plane inverse)
 template <int DL, int G> __device__ __forceinline__ int plane_of_rank(int r) { return (r % DL) * G + r / DL; }
+
+// Pair mode (G == 2, MP_CTAB_PAIR): the upper lane of a cell negates its distances before the
+// in-lane sort, so after the sort it holds its run negated and reversed.  The cross-lane bitonic
+// "flip" then pairs equal register indices and is the same instruction in both lanes,
+// s = min(s, -partner(s)): one SHFL + one FMNMX per element and no lane-dependent min / max (which
+// costs FMNMX + predicated FMNMX), and the in-lane half-cleaners stay ascending in both lanes.
+// Padded dims have D = 0 exactly (a = 1, QT = 2m) and sort FIRST: sorted index si = rank + npad.
+// After the fused scan of the stored values P_g, lane 0 register j holds S at sorted index j;
+// lane 1 register j <= DL - 2 holds sorted index 2 DL - 2 - j (= c_1 + P_1[j] with
+// c_1 = P_0[DL - 1] - P_1[DL - 1]) and register DL - 1 the total (sorted index 2 DL - 1).
+template <int DL> __device__ __forceinline__ int pair_si(int g, int kk) {
+    return g == 0 ? kk : (kk == DL - 1 ? 2 * DL - 1 : 2 * DL - 2 - kk);
+}
+// position of sorted index si in the per-slot threshold array: lane g's registers are contiguous
+template <int DL> __device__ __forceinline__ int pair_pos_of_si(int si) {
+    return si < DL ? si : (si == 2 * DL - 1 ? 2 * DL - 1 : 3 * DL - 2 - si);
+}
 
 template <int DL, int G, int NT, bool SELF>
 __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32) mp_diag_ctab(const MainParams p) {
@@ -116,6 +141,7 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
     using K = unsigned long long;
     constexpr int D = Cg::D, NCC = Cg::NCC, RR = Cg::RR, RC = Cg::RC, SS = Cg::SS, SB = Cg::SB;
     constexpr int NTHR = Cg::NTHR;
+    constexpr bool PM = MP_CTAB_PAIR && MP_CTAB_TA && G == 2;   // pair mode (pair_si)
     constexpr int FOLD = SB > MP_FOLD ? SB : MP_FOLD;
 
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -140,15 +166,18 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
     const int tid = threadIdx.x;
     const int c = tid / G, g = tid & (G - 1);  // cell of the block tile, lane within the cell
     const unsigned stat_bytes = (unsigned)d * 16u;
+    const int npad = D - d;
+    // padded planes: pair mode D = 0 (a = 1, QT = 2m; sorts first), else D ~ 1e18 (sorts last)
+    const float pad_a = PM ? 1.f : PT<float>::pad_a();
 
     // padded planes [d, D) never change (TMA writes planes [0, d) of a slot): set them once
     for (int e = tid; e < (RR + RC) * (D - d); e += NT) {
         const int sl = e / (D - d), pl = d + e % (D - d);
         V4* dst = (sl < RR ? rowv + (size_t)sl * SS : colv + (size_t)(sl - RR) * SS) + pl;
-        *dst = make_float4(0.f, 0.f, PT<float>::pad_a(), NINF);
+        *dst = make_float4(0.f, 0.f, pad_a, NINF);
     }
     if (tid == 0) {
-        mbar_init(bar, 1);
+        mbar_init(bar, 1);   // thread 0 arrives once per batch (issue_batch)
         fence_proxy_async();
     }
     unsigned phase = 0;
@@ -183,7 +212,7 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
             const int pos = C0 + q;
             if (pos >= 0 && pos < n32) continue;
             V4* dst = colv + (size_t)cslot(pos) * SS;
-            for (int pl = tid; pl < D; pl += NT) dst[pl] = make_float4(0.f, 0.f, PT<float>::pad_a(), NINF);
+            for (int pl = tid; pl < D; pl += NT) dst[pl] = make_float4(0.f, 0.f, pad_a, NINF);
         }
     };
     // threshold words of the staged positions: entry e = (position index, rank r); rank r's
@@ -192,12 +221,14 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
     // (dst: float index of the threshold word in the rings)
     float* const ringf = reinterpret_cast<float*>(smem_raw);
     auto thr_entry = [&](int e, int R0, int r_lo, int nr, int C0, int c_lo, int& dst) -> float {
-        const int pi = e / D, r = e - pi * D;
+        const int pi = e / D, q = e - pi * D;   // q: rank (pair mode: sorted index, rank q - npad)
         const bool is_row = pi < nr;
         const int pos = is_row ? R0 + r_lo + pi : C0 + c_lo + (pi - nr);
         const int slot = is_row ? rslot(pos) : RR + cslot(pos);
-        dst = (slot * SS + plane_of_rank<DL, G>(r)) * 4 + 3;
-        if (r >= d || pos < 0 || pos >= n32) return NINF;
+        if (MP_CTAB_TA) dst = (int)(Cg::stat_ring_bytes / 4) + slot * D + (PM ? pair_pos_of_si<DL>(q) : q);
+        else dst = (slot * SS + plane_of_rank<DL, G>(q)) * 4 + 3;
+        const int r = PM ? q - npad : q;
+        if (r < 0 || r >= d || pos < 0 || pos >= n32) return NINF;
         return __uint_as_float(__ldcg(reinterpret_cast<const unsigned*>(keys + (size_t)pos * d + r) + 1));
     };
 
@@ -258,7 +289,7 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
 #pragma unroll
                 for (int kk = 0; kk < SC; ++kk) {  // lane g's register c0 + kk is dim (c0 + kk) G + g
                     const bool pad = ((c0 + kk) * G + g) >= d;
-                    QT[c0 + kk] = pad ? -1.f : acc[kk];
+                    QT[c0 + kk] = pad ? (PM ? two_m : -1.f) : acc[kk];
                     QL[c0 + kk] = pad ? 0.f : -cmp[kk];
                 }
             }
@@ -267,7 +298,7 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
             seed_cell(lo);
         } else {
 #pragma unroll
-            for (int kk = 0; kk < DL; ++kk) { QT[kk] = (kk * G + g) >= d ? -1.f : 0.f; QL[kk] = 0.f; }
+            for (int kk = 0; kk < DL; ++kk) { QT[kk] = (kk * G + g) >= d ? (PM ? two_m : -1.f) : 0.f; QL[kk] = 0.f; }
         }
 
         // first batch landed: patch its thresholds directly (once per tile)
@@ -324,9 +355,14 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
                 const int row = R0 + s, col = row + dlt;
                 const bool active = row >= lo32 && row < hi32;
                 const bool upd = row > lo32 && row < hi32 && s != seeded_step;
-                const V4* Rs = rowv + (size_t)rslot(row) * SS;
-                const V4* Cs = colv + (size_t)cslot(C0 + s + c) * SS;
-                float S[DL], thr[DL];
+                const int sr = rslot(row), sc = cslot(C0 + s + c);
+                const V4* Rs = rowv + (size_t)sr * SS;
+                const V4* Cs = colv + (size_t)sc * SS;
+                // thresholds of this lane's ranks g DL .. g DL + DL - 1 (MP_CTAB_TA)
+                float* TRs = ringf + Cg::stat_ring_bytes / 4 + (size_t)sr * D + g * DL;
+                float* TCs = ringf + Cg::stat_ring_bytes / 4 + (size_t)(RR + sc) * D + g * DL;
+                float S[DL];
+                [[maybe_unused]] float thr[MP_CTAB_TA ? 1 : DL];
 #pragma unroll
                 for (int kk = 0; kk < DL; ++kk) {
                     const int pl = kk * G + g;
@@ -337,12 +373,34 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
                     S[kk] = PT<float>::sqrt_abs(fmaf(-QL[kk], pr, fmaf(-QT[kk], pr, two_m)));  // Eq. (1)
                     // plane kk G + g carries the threshold of rank g DL + kk: the rank this
                     // lane holds at register kk after the sort (one test covers row and column)
-                    thr[kk] = SELF ? fmaxf(R.w, C.w) : R.w;
+                    if constexpr (!MP_CTAB_TA) thr[kk] = SELF ? fmaxf(R.w, C.w) : R.w;
+                }
+                if constexpr (PM) {
+                    const float sgn = g ? -1.f : 1.f;
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) S[kk] *= sgn;
                 }
                 sort_net<float, DL>(S);                                                  // Eq. (2)
+                if constexpr (PM) {
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) S[kk] = fminf(S[kk], -__shfl_xor_sync(FULL, S[kk], 1));
+#pragma unroll
+                    for (int dist = DL / 2; dist >= 2; dist >>= 1)
+#pragma unroll
+                        for (int kk = 0; kk < DL; ++kk)
+                            if ((kk & dist) == 0) cswap(S[kk], S[kk + dist]);
+                    pair_scan<float, DL>(S);                                             // Eq. (2) scan
+                    const float tot = S[DL - 1];
+                    const float oth = __shfl_xor_sync(FULL, tot, 1);
+                    const float cg = g ? oth - tot : 0.f;
+#pragma unroll
+                    for (int kk = 0; kk < DL - 1; ++kk) S[kk] += cg;
+                    S[DL - 1] = g ? cg : tot;
+                } else {
                 if constexpr (G > 1) lane_merge<float, DL, G, true>(S, g);
                 pair_scan<float, DL>(S);                                                 // Eq. (2) scan
-                if constexpr (G > 1) {
+                }
+                if constexpr (G > 1 && !PM) {
                     float tot = S[DL - 1];
 #pragma unroll
                     for (int dd = 1; dd < G; dd <<= 1) {
@@ -356,22 +414,33 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
                 }
                 bool h[4] = {false, false, false, false};
 #pragma unroll
-                for (int kk = 0; kk < DL; ++kk) h[kk & 3] |= S[kk] <= thr[kk];
+                for (int kk = 0; kk < DL; kk += 4) {
+                    if constexpr (MP_CTAB_TA) {
+                        const float4 tr = *reinterpret_cast<const float4*>(TRs + kk);
+                        h[0] |= S[kk] <= tr.x; h[1] |= S[kk + 1] <= tr.y; h[2] |= S[kk + 2] <= tr.z; h[3] |= S[kk + 3] <= tr.w;
+                        if (SELF) {
+                            const float4 tc = *reinterpret_cast<const float4*>(TCs + kk);
+                            h[0] |= S[kk] <= tc.x; h[1] |= S[kk + 1] <= tc.y; h[2] |= S[kk + 2] <= tc.z; h[3] |= S[kk + 3] <= tc.w;
+                        }
+                    } else {
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) h[q] |= S[kk + q] <= thr[kk + q];
+                    }
+                }
                 if (((h[0] | h[1]) | (h[2] | h[3])) && active) {
                     // Eq. (3), write-through: merge into the global key, lower the hint
 #pragma unroll
                     for (int kk = 0; kk < DL; ++kk) {
                         const float v = S[kk];
-                        if (!(v <= thr[kk])) continue;
-                        const int pl = kk * G + g, rk = g * DL + kk;
+                        const int pl = kk * G + g, rk = PM ? pair_si<DL>(g, kk) - npad : g * DL + kk;
                         const unsigned vb = __float_as_uint(v);
-                        float* rw = const_cast<float*>(&Rs[pl].w);
+                        float* rw = MP_CTAB_TA ? TRs + kk : const_cast<float*>(&Rs[pl].w);
                         if (v <= *reinterpret_cast<volatile float*>(rw)) {
                             atomicMin(keys + (size_t)row * d + rk, ((K)vb << 32) | (unsigned)col);
                             atomicMin(reinterpret_cast<unsigned*>(rw), vb);
                         }
                         if (SELF) {
-                            float* cw = const_cast<float*>(&Cs[pl].w);
+                            float* cw = MP_CTAB_TA ? TCs + kk : const_cast<float*>(&Cs[pl].w);
                             if (v <= *reinterpret_cast<volatile float*>(cw)) {
                                 atomicMin(keys + (size_t)col * d + rk, ((K)vb << 32) | (unsigned)row);
                                 atomicMin(reinterpret_cast<unsigned*>(cw), vb);
