@@ -143,6 +143,26 @@ mp_status mp_plan_diagonals(int64_t d, int64_t n, int64_t m, mp_precision prec, 
  * events around the main diagonal kernel only) and its launch count. */
 mp_status mp_last_timing(const mp_ctx* ctx, double* main_kernel_ms, int64_t* launches);
 
+/*
+ * Stage self-tests (per-stage unit tests of SURVEY 4; tests/test_gpu_stages.py).  They run ONE
+ * stage of the hot path on the device with the same device code the fused kernels use, on host
+ * buffers (copies in and out included), so a stage can be checked against the oracle / numpy in
+ * isolation.  Not part of the compute path.
+ *
+ * mp_selftest_sort_scan: for each of `count` cells, the FP32 kernel variant chosen for `d`
+ *   (warp tiles for d <= 32, block-cooperative tiles above: the same sort network, cross-lane
+ *   merge and fused scan templates) sorts the cell's d values ascending and writes the inclusive
+ *   prefix sums S_k = sum of the k+1 smallest (Eq. 2).  in / out: count x d
+ *   floats, cell-major.  Values may be any non-negative float, +inf or denormal.
+ * mp_selftest_precompute: the precalculation of mode `prec` (readings G7,
+ *   R1') on T (d x L, L = n + m - 1): writes df, dg, a (each n x d, position-major, as doubles;
+ *   half modes: the unscaled values divided back by the per-dimension power-of-two scale are NOT
+ *   returned -- FP64 and FP32 only).
+ */
+mp_status mp_selftest_sort_scan(mp_ctx* ctx, int64_t d, int64_t count, const float* in, float* out);
+mp_status mp_selftest_precompute(mp_ctx* ctx, const double* T, int64_t d, int64_t n, int64_t m,
+                                 mp_precision prec, double* df, double* dg, double* a);
+
 #ifdef __cplusplus
 }
 #endif

@@ -1,11 +1,15 @@
 """Build libmstamp_b200.so for sm_100a (in-tree, so the .so travels with the repo snapshot).
 
-The kernel templates are instantiated in several translation units compiled in
-parallel (csrc/inst_*.cu are generated here), then linked with the host ABI.
+The kernel templates are instantiated in several translation units (csrc/inst_*.cu, committed:
+one explicit instantiation each) compiled in parallel, then linked with the host ABI.  The
+library is rebuilt whenever the sources, headers or flags differ from the ones it was built
+from: a content hash is stored next to it (lib/libmstamp_b200.so.sha256), so a shipped tree
+with a stale library (timestamps do not travel reliably) is rebuilt, not reused.
 """
 from __future__ import annotations
 
 import concurrent.futures as cf
+import hashlib
 import os
 import subprocess
 import sys
@@ -31,11 +35,25 @@ def _deps():
     return [os.path.join(CSRC, f) for f in os.listdir(CSRC)]
 
 
+HASH = LIB + ".sha256"
+
+
+def _digest():
+    h = hashlib.sha256()
+    h.update(" ".join([NVCC] + ARCH + FLAGS).encode())
+    inc = os.path.join(HERE, "..", "include")
+    for f in sorted(_deps()) + sorted(os.path.join(inc, x) for x in os.listdir(inc)):
+        h.update(os.path.basename(f).encode())
+        with open(f, "rb") as fh:
+            h.update(fh.read())
+    return h.hexdigest()
+
+
 def _stale():
-    if not os.path.exists(LIB):
+    if not os.path.exists(LIB) or not os.path.exists(HASH):
         return True
-    t = os.path.getmtime(LIB)
-    return any(os.path.getmtime(f) > t for f in _deps())
+    with open(HASH) as f:
+        return f.read().strip() != _digest()
 
 
 def _compile(src):
@@ -57,6 +75,8 @@ def build(force: bool = False, verbose: bool = True) -> str:
         objs = list(ex.map(_compile, srcs))
     cmd = [NVCC] + ARCH + ["-shared", "-o", LIB] + objs + ["-lcudart"]
     subprocess.check_call(cmd)
+    with open(HASH, "w") as f:
+        f.write(_digest() + "\n")
     if verbose:
         print(f"built {LIB}", file=sys.stderr)
     return LIB

@@ -480,6 +480,59 @@ mp_status mp_compute(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, 
     return MP_OK;
 }
 
+mp_status mp_selftest_sort_scan(mp_ctx* ctx, int64_t d, int64_t count, const float* in, float* out) {
+    if (!ctx || !in || !out || d < 1 || d > MP_MAX_D || count < 1) return fail(ctx, MP_ERR_INVALID, "bad arguments");
+    MP_CUDA(ctx, cudaSetDevice(ctx->device));
+    cudaStream_t s = ctx->stream;
+    Buf a, b;
+    const size_t bytes = (size_t)count * d * sizeof(float);
+    MP_CUDA(ctx, ensure(a, bytes));
+    cudaError_t e = ensure(b, bytes);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(a.p, in, bytes, cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess) e = mpk::launch_selftest_sort_scan((int)d, count, (const float*)a.p, (float*)b.p, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(out, b.p, bytes, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    release(a);
+    release(b);
+    return e == cudaSuccess ? MP_OK : cuda_fail(ctx, e, "mp_selftest_sort_scan");
+}
+
+mp_status mp_selftest_precompute(mp_ctx* ctx, const double* T, int64_t d, int64_t n, int64_t m,
+                                 mp_precision prec, double* df, double* dg, double* a) {
+    if (!ctx) return MP_ERR_INVALID;
+    mp_status st = validate(ctx, T, d, n, m, prec);
+    if (st != MP_OK) return st;
+    if (!df || !dg || !a || (prec != MP_FP64 && prec != MP_FP32)) return fail(ctx, MP_ERR_INVALID, "bad arguments");
+    MP_CUDA(ctx, cudaSetDevice(ctx->device));
+    cudaStream_t s = ctx->stream;
+    const int64_t L = n + m - 1;
+    MP_CUDA(ctx, ensure(ctx->dT, (size_t)d * L * 8));
+    MP_CUDA(ctx, cudaMemcpyAsync(ctx->dT.p, T, (size_t)d * L * 8, cudaMemcpyHostToDevice, s));
+    const mpk::Variant var = mpk::pick_variant(prec, (int)d);
+    mpk::PreParams pp{};
+    pp.n = n; pp.d = (int)d; pp.m = (int)m; pp.Dp = var.DL * var.G;
+    if (var.ctab) { pp.pm_G = var.G; pp.pm_DL = var.DL; }
+    const size_t eb = elt_bytes(prec), tbs = 8;
+    MP_CUDA(ctx, ensure(ctx->nrm, (size_t)n * d * tbs));
+    pp.nrm32 = (float*)ctx->nrm.p; pp.nrm64 = (double*)ctx->nrm.p;
+    MP_CUDA(ctx, ensure(ctx->st_q, (size_t)n * d * 4 * eb));
+    MP_CUDA(ctx, ensure(ctx->mu_q, (size_t)n * d * tbs));
+    MP_CUDA(ctx, ensure(ctx->mup_q, (size_t)n * pp.Dp * eb));
+    MP_CUDA(ctx, ensure(ctx->tw_q, (size_t)L * pp.Dp * eb));
+    pp.T = (const double*)ctx->dT.p; pp.st = ctx->st_q.p; pp.mu = ctx->mu_q.p; pp.mup = ctx->mup_q.p; pp.tw = ctx->tw_q.p;
+    MP_CUDA(ctx, mpk::launch_precompute(prec, pp, s));
+    Buf o;
+    MP_CUDA(ctx, ensure(o, (size_t)n * d * 3 * 8));
+    double* od = (double*)o.p;
+    cudaError_t e = mpk::launch_selftest_unpack(prec, ctx->st_q.p, n, (int)d, od, od + n * d, od + 2 * n * d, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(df, od, (size_t)n * d * 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(dg, od + n * d, (size_t)n * d * 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(a, od + 2 * n * d, (size_t)n * d * 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    release(o);
+    return e == cudaSuccess ? MP_OK : cuda_fail(ctx, e, "mp_selftest_precompute");
+}
+
 mp_status mp_last_timing(const mp_ctx* ctx, double* main_kernel_ms, int64_t* launches) {
     if (!ctx || !main_kernel_ms || !launches) return MP_ERR_INVALID;
     *launches = ctx->last_launches;

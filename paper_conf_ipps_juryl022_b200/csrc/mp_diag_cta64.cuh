@@ -50,6 +50,10 @@ namespace mpk {
 #ifndef MP_CTA64_QN
 #define MP_CTA64_QN 256   // per-block queue of global write-through merges, flushed once per batch (0: off)
 #endif
+#ifndef MP_CTA64_TA
+#define MP_CTA64_TA 1   // FP32 filter thresholds in rank-contiguous per-slot arrays, read as vectors after the
+                        // scan (none live through the sort: -32 registers), instead of the entries' thr word
+#endif
 #ifndef MP_CTA64_ROWKEY
 #define MP_CTA64_ROWKEY 1   // row bests in a shared-memory key ring (d <= 256), merged at eviction
 #endif
@@ -93,7 +97,11 @@ template <int DL, int G, int NW> struct CtaGeo64 {
     static constexpr int RR = 3 * SB;
     static constexpr int RC = 3 * SB + NCC - 1;
     static constexpr bool ROWKEY = CtaShape64<G>::ROWKEY;
-    static constexpr size_t bytes = (size_t)(RR + RC) * D * sizeof(E64) + (ROWKEY ? (size_t)RR * D * sizeof(K64) + 16 * ((RR * 4 + 15) / 16) : 0) + (size_t)MP_CTA64_QN * sizeof(PendQ) + 32;
+    static constexpr size_t base_bytes = (size_t)(RR + RC) * D * sizeof(E64) + (ROWKEY ? (size_t)RR * D * sizeof(K64) + 16 * ((RR * 4 + 15) / 16) : 0) + (size_t)MP_CTA64_QN * sizeof(PendQ) + 32;
+    // threshold arrays where they fit next to the rings (not at d = 512)
+    static constexpr bool TA = MP_CTA64_TA && base_bytes + (size_t)(RR + RC) * D * 4 <= 227 * 1024;
+    static constexpr size_t ta_bytes = TA ? (size_t)(RR + RC) * D * 4 : 0;   // [slot][rank] float
+    static constexpr size_t bytes = base_bytes + ta_bytes;
 };
 
 template <int DL, int G, int NW, bool SELF>
@@ -106,6 +114,7 @@ mp_diag_cta64(const MainParams p) {
 
     extern __shared__ __align__(16) unsigned char smem_raw[];
     constexpr bool ROWKEY = Cg::ROWKEY;
+    constexpr bool TA = Cg::TA;
     E64* rowv = reinterpret_cast<E64*>(smem_raw);
     E64* colv = rowv + (size_t)RR * D;
     K64* rowk = reinterpret_cast<K64*>(colv + (size_t)RC * D);                      // ROWKEY: [RR][D]
@@ -114,6 +123,7 @@ mp_diag_cta64(const MainParams p) {
     PendQ* pq = reinterpret_cast<PendQ*>(reinterpret_cast<unsigned char*>(rdirty) + (ROWKEY ? 16 * ((RR * 4 + 15) / 16) : 0));
     long long* tile_sh = reinterpret_cast<long long*>(pq + QN);
     unsigned* qn = reinterpret_cast<unsigned*>(tile_sh + 1);   // queued merges (monotone)
+    float* ta = reinterpret_cast<float*>(tile_sh + 4);           // MP_CTA64_TA: thresholds [slot][rank], rows then columns
 
     const double4* __restrict__ st_q = reinterpret_cast<const double4*>(p.st_q);
     const double4* __restrict__ st_r = reinterpret_cast<const double4*>(p.st_r);
@@ -205,8 +215,11 @@ mp_diag_cta64(const MainParams p) {
         for (int e = tid; e < cnt * D; e += NT) {
             const int pi = e / D, pl = e - pi * D;
             const int pos = base + p_lo + pi;
-            E64& en = buf[(is_row ? rslot(pos) : cslot(pos)) * D + pl];
-            en.thr = __double2float_ru(*reinterpret_cast<const double*>(&en.thr) * margin);
+            const int sl = is_row ? rslot(pos) : cslot(pos);
+            E64& en = buf[sl * D + pl];
+            const float t = __double2float_ru(*reinterpret_cast<const double*>(&en.thr) * margin);
+            if (TA) ta[(is_row ? sl : RR + sl) * D + rank_of_plane<DL, G>(pl)] = t;
+            else en.thr = t;
         }
     };
 
@@ -302,8 +315,10 @@ mp_diag_cta64(const MainParams p) {
                 // ---- filter path: FP64 recurrence + D^2, FP32 distance / sort / scan / compare
                 float Sf[DL];
                 bool h[4] = {false, false, false, false};
+                float* TRs = ta + (size_t)sr * D + g * DL;          // this lane's ranks g DL ..
+                float* TCs = ta + (size_t)(RR + sc) * D + g * DL;
                 {
-                    float trf[DL], tcf[DL];
+                    [[maybe_unused]] float trf[TA ? 1 : DL], tcf[TA ? 1 : DL];
 #pragma unroll
                     for (int kk = 0; kk < DL; ++kk) {
                         const int pl = kk * G + g;
@@ -312,8 +327,7 @@ mp_diag_cta64(const MainParams p) {
                         if (upd) QT[kk] = fma(R.df, C.dg, fma(C.df, R.dg, QT[kk]));      // Eq. (1)
                         const double d2 = fma(-QT[kk], R.a * C.a, two_m);
                         Sf[kk] = sqrt_abs_f(__double2float_rn(d2));
-                        trf[kk] = R.thr;
-                        tcf[kk] = C.thr;
+                        if constexpr (!TA) { trf[kk] = R.thr; tcf[kk] = C.thr; }
                     }
                     sort_net<float, DL>(Sf);
                     lane_merge<float, DL, G>(Sf, g);
@@ -328,10 +342,23 @@ mp_diag_cta64(const MainParams p) {
                     float excl = __shfl_up_sync(FULL, tot, 1, G);
                     if (g == 0) excl = 0.f;
 #pragma unroll
-                    for (int kk = 0; kk < DL; ++kk) {
-                        Sf[kk] += excl;
-                        h[kk & 3] |= Sf[kk] <= trf[kk];
-                        if (SELF) h[kk & 3] |= Sf[kk] <= tcf[kk];
+                    for (int kk = 0; kk < DL; ++kk) Sf[kk] += excl;
+#pragma unroll
+                    for (int kk = 0; kk < DL; kk += 4) {
+                        if constexpr (TA) {
+                            const float4 tr = *reinterpret_cast<const float4*>(TRs + kk);
+                            h[0] |= Sf[kk] <= tr.x; h[1] |= Sf[kk + 1] <= tr.y; h[2] |= Sf[kk + 2] <= tr.z; h[3] |= Sf[kk + 3] <= tr.w;
+                            if (SELF) {
+                                const float4 tc = *reinterpret_cast<const float4*>(TCs + kk);
+                                h[0] |= Sf[kk] <= tc.x; h[1] |= Sf[kk + 1] <= tc.y; h[2] |= Sf[kk + 2] <= tc.z; h[3] |= Sf[kk + 3] <= tc.w;
+                            }
+                        } else {
+#pragma unroll
+                            for (int q4 = 0; q4 < 4; ++q4) {
+                                h[q4] |= Sf[kk + q4] <= trf[kk + q4];
+                                if (SELF) h[q4] |= Sf[kk + q4] <= tcf[kk + q4];
+                            }
+                        }
                     }
                 }
                 const bool hit = ((h[0] | h[1]) | (h[2] | h[3])) && active;
@@ -370,7 +397,7 @@ mp_diag_cta64(const MainParams p) {
                     for (int qq = 0; qq + 1 < DL; ++qq) S[qq] = S[qq + 1];
                     const int rk = rank_of_plane<DL, G>(pl);
                     if (rk >= d) continue;
-                    float& thr_r = rowv[sr * D + pl].thr;
+                    float& thr_r = TA ? TRs[kk] : rowv[sr * D + pl].thr;
                     if (v <= (double)thr_r) {
                         if constexpr (ROWKEY) {
                             smem_merge64(&rowk[sr * D + pl], v, (unsigned)col);
@@ -381,7 +408,7 @@ mp_diag_cta64(const MainParams p) {
                         thr_r = fminf(thr_r, __double2float_ru(v * margin));
                     }
                     if (SELF) {
-                        float& thr_c = colv[sc * D + pl].thr;
+                        float& thr_c = TA ? TCs[kk] : colv[sc * D + pl].thr;
                         if (v <= (double)thr_c) {
                             merge_q((size_t)col * d + rk, v, (unsigned)row);
                             thr_c = fminf(thr_c, __double2float_ru(v * margin));

@@ -75,5 +75,9 @@ cudaError_t launch_keys_to_ext(int prec, const void* keys, void* ext, long long 
                                cudaStream_t s);
 cudaError_t launch_key_mask(long long count, long long* ext, const long long* gv, cudaStream_t s);
 cudaError_t launch_check_finite(const double* x, long long count, int* flag, cudaStream_t s);
+// stage self-tests (include/mp.h)
+cudaError_t launch_selftest_sort_scan(int d, long long count, const float* in, float* out, cudaStream_t s);
+cudaError_t launch_selftest_unpack(int prec, const void* st, long long n, int d, double* df, double* dg, double* a,
+                                   cudaStream_t s);
 
 }  // namespace mpk

@@ -558,6 +558,91 @@ cudaError_t launch_finalize(int prec, const void* keys_ext, long long n, int d, 
     return cudaGetLastError();
 }
 
+// ------------------------------------------------------------------ stage self-tests
+// One cell per G lanes, DL values per lane, exactly as the fused kernels hold them: lane g's
+// register kk is dim kk G + g; the sort / merge / scan templates are the kernels' own.
+template <int DL, int G, bool CTAB>
+__global__ void selftest_sort_scan(int d, long long count, const float* in, float* out) {
+    constexpr int CPW = 32 / G;  // cells per warp
+    const long long cell = (blockIdx.x * (long long)blockDim.x + threadIdx.x) / G;
+    const int g = threadIdx.x & (G - 1);
+    const bool ok = cell < count;   // whole warps stay converged for the shuffles
+    (void)CPW;
+    float S[DL];
+#pragma unroll
+    for (int kk = 0; kk < DL; ++kk) {
+        const int dim = kk * G + g;
+        S[kk] = (ok && dim < d) ? in[cell * d + dim] : PT<float>::pad_a();   // padded dims sort last
+    }
+    if constexpr (G == 1 && DL >= 8 && last_layer_adjacent<DL>()) {
+        sort_scan_fused<float, DL>(S);        // mp_diag, one lane per cell
+    } else if constexpr (G == 1) {
+        sort_net<float, DL>(S);
+#pragma unroll
+        for (int kk = 1; kk < DL; ++kk) S[kk] += S[kk - 1];
+    } else {
+        sort_net<float, DL>(S);
+        if constexpr (CTAB) {                 // mp_diag_ctab: last merge layer fused into the scan
+            lane_merge<float, DL, G, true>(S, g);
+            pair_scan<float, DL>(S);
+        } else {                              // mp_diag, G lanes per cell: two half chains
+            lane_merge<float, DL, G>(S, g);
+#pragma unroll
+            for (int kk = 1; kk < DL / 2; ++kk) S[kk] += S[kk - 1];
+#pragma unroll
+            for (int kk = DL / 2 + 1; kk < DL; ++kk) S[kk] += S[kk - 1];
+#pragma unroll
+            for (int kk = DL / 2; kk < DL; ++kk) S[kk] += S[DL / 2 - 1];
+        }
+        float tot = S[DL - 1];
+#pragma unroll
+        for (int dd = 1; dd < G; dd <<= 1) {
+            const float y = __shfl_up_sync(FULL, tot, dd, G);
+            if (g >= dd) tot += y;
+        }
+        float excl = __shfl_up_sync(FULL, tot, 1, G);
+        if (g == 0) excl = 0.f;
+#pragma unroll
+        for (int kk = 0; kk < DL; ++kk) S[kk] += excl;
+    }
+#pragma unroll
+    for (int kk = 0; kk < DL; ++kk) {
+        const int rk = g * DL + kk;   // lane g holds ranks g DL .. g DL + DL - 1
+        if (ok && rk < d) out[cell * d + rk] = S[kk];
+    }
+}
+
+cudaError_t launch_selftest_sort_scan(int d, long long count, const float* in, float* out, cudaStream_t s) {
+    const Variant v = pick_variant(P32, d);
+    const long long threads = count * v.G;
+    const unsigned grid = (unsigned)((threads + 127) / 128);
+#define MP_STCASE(dl, g, ct)                                                                 \
+    if (v.DL == dl && v.G == g && v.ctab == ct) {                                            \
+        selftest_sort_scan<dl, g, ct><<<grid, 128, 0, s>>>(d, count, in, out);               \
+        return cudaGetLastError();                                                           \
+    }
+    MP_STCASE(1, 1, false) MP_STCASE(2, 1, false) MP_STCASE(4, 1, false) MP_STCASE(8, 1, false)
+    MP_STCASE(16, 1, false) MP_STCASE(16, 2, false) MP_STCASE(16, 4, true) MP_STCASE(16, 8, true)
+    MP_STCASE(16, 16, true) MP_STCASE(16, 32, true) MP_STCASE(32, 32, true) MP_STCASE(32, 2, true)
+    MP_STCASE(32, 4, true) MP_STCASE(32, 8, true) MP_STCASE(32, 16, true)
+#undef MP_STCASE
+    return cudaErrorInvalidValue;
+}
+
+template <class T>
+__global__ void selftest_unpack(const typename PT<T>::V4* st, long long count, double* df, double* dg, double* a) {
+    const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (i < count) { df[i] = (double)st[i].x; dg[i] = (double)st[i].y; a[i] = (double)st[i].z; }
+}
+cudaError_t launch_selftest_unpack(int prec, const void* st, long long n, int d, double* df, double* dg, double* a,
+                                   cudaStream_t s) {
+    const long long cnt = n * d;
+    if (prec == P64) selftest_unpack<double><<<grid1d(cnt, 256), 256, 0, s>>>(reinterpret_cast<const double4*>(st), cnt, df, dg, a);
+    else if (prec == P32) selftest_unpack<float><<<grid1d(cnt, 256), 256, 0, s>>>(reinterpret_cast<const float4*>(st), cnt, df, dg, a);
+    else return cudaErrorInvalidValue;
+    return cudaGetLastError();
+}
+
 cudaError_t launch_check_finite(const double* x, long long count, int* flag, cudaStream_t s) {
     check_finite<<<1184, 256, 0, s>>>(x, count, flag);
     return cudaGetLastError();

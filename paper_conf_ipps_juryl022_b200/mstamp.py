@@ -23,7 +23,8 @@ STATUS = {0: "MP_OK", 1: "MP_ERR_INVALID", 2: "MP_ERR_NOMEM", 3: "MP_ERR_CUDA", 
           5: "MP_ERR_UNSUPPORTED"}
 EXPORTS = ["mp_init", "mp_free", "mp_last_error", "mp_version", "mp_compute", "mp_compute_device",
            "mp_key_words", "mp_partial_device", "mp_key_mask_device", "mp_finalize_device",
-           "mp_plan_bands", "mp_plan_diagonals", "mp_last_timing"]
+           "mp_plan_bands", "mp_plan_diagonals", "mp_last_timing", "mp_selftest_sort_scan",
+           "mp_selftest_precompute"]
 
 _lib = None
 
@@ -73,6 +74,10 @@ def load():
     lib.mp_plan_diagonals.restype = i32
     lib.mp_last_timing.argtypes = [p, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(i64)]
     lib.mp_last_timing.restype = i32
+    lib.mp_selftest_sort_scan.argtypes = [p, i64, i64, p, p]
+    lib.mp_selftest_sort_scan.restype = i32
+    lib.mp_selftest_precompute.argtypes = [p, p, i64, i64, i64, i32, p, p, p]
+    lib.mp_selftest_precompute.restype = i32
     _lib = lib
     return lib
 
@@ -249,6 +254,29 @@ class Context:
         st = load().mp_finalize_device(self._ctx, ctypes.c_void_p(s.cuda_stream), d, n, _prec(prec),
                                        _tptr(keys), _tptr(P), _tptr(I))
         self._check(st, "mp_finalize_device")
+
+    # ---- stage self-tests (include/mp.h; tests only)
+    def selftest_sort_scan(self, X):
+        """X (count, d) float32 -> inclusive prefix sums of each row sorted ascending, computed by
+        the FP32 kernels' own sort / merge / scan device code for this d."""
+        X = np.ascontiguousarray(X, dtype=np.float32)
+        count, d = X.shape
+        out = np.empty_like(X)
+        st = load().mp_selftest_sort_scan(self._ctx, d, count, X.ctypes.data_as(ctypes.c_void_p),
+                                          out.ctypes.data_as(ctypes.c_void_p))
+        self._check(st, "mp_selftest_sort_scan")
+        return out
+
+    def selftest_precompute(self, T, m, prec="fp64"):
+        """(df, dg, a), each (n, d) position-major, from the device precalculation of mode prec."""
+        T = np.ascontiguousarray(T, dtype=np.float64)
+        d, L = T.shape
+        n = L - m + 1
+        outs = [np.empty((n, d)) for _ in range(3)]
+        st = load().mp_selftest_precompute(self._ctx, T.ctypes.data_as(ctypes.c_void_p), d, n, m, _prec(prec),
+                                           *[o.ctypes.data_as(ctypes.c_void_p) for o in outs])
+        self._check(st, "mp_selftest_precompute")
+        return tuple(outs)
 
     def last_timing(self):
         ms = ctypes.c_double()
