@@ -346,8 +346,13 @@ def main():
                          "'auto'), 'properties' checks bound / monotonicity / planted motif (larger configs)")
     ap.add_argument("--backend", default="nccl", help="process-group backend for N>1 (gloo: functional "
                     "test of the multi-rank path, e.g. several ranks on one GPU via MP_BENCH_DEVICE)")
+    ap.add_argument("--dry-run", action="store_true",
+                    help="functional run of the multi-rank path: one step, no warm-up; the line says "
+                         "dry_run and is not a bench value")
     args = ap.parse_args()
-    args.warmup = max(args.warmup, 3)
+    args.warmup = 0 if args.dry_run else max(args.warmup, 3)
+    if args.dry_run:
+        args.steps = 1
     world = int(os.environ.get("WORLD_SIZE", "1"))
     if args.config is None:
         args.config = "C3" if world == 1 else "C4"
@@ -561,6 +566,8 @@ def main():
                 "per_config_band": per_cfg or None, "computed_cells_per_s": cells * d / (ms * 1e-3)}
         if merge_check is not None:
             line["merge_check"] = merge_check
+        if args.dry_run:
+            line["dry_run"] = True
         print(json.dumps(line), flush=True)
     ctx.close()
     if world > 1:

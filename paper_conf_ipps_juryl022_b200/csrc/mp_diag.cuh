@@ -795,6 +795,7 @@ mp_diag(const MainParams p) {
                         need_c = __any_sync(FULL, need_c);
                     }
                     if (!need_r && !need_c) return;
+                    __syncwarp();   // every lane read the ring bests before a leader updates them
                     // row group: W cells per lane x CA lanes
                     T vr = v[0];
 #pragma unroll
@@ -844,6 +845,7 @@ mp_diag(const MainParams p) {
                             }
                         }
                     }
+                    __syncwarp();   // the leaders' ring updates are visible to the next rank's reads
                 };
                 if constexpr (MP_SLOW_UNROLL) {
                     // ranks some lane can improve, from registers (S stays live; the ring's
@@ -938,6 +940,7 @@ mp_diag(const MainParams p) {
             row_out = rx;
             evict(false, C0, col_out, s0);
             col_out = s0;
+            __syncwarp();   // every eviction read its ring slot before a prefetch can overwrite it
             const int nxt = min(s0 + 2 * SB, s_end);
             const int r_need = min(nxt, nrows), c_need = nxt + CW - 1;
             stage(true, R0, row_in, r_need);

@@ -23,6 +23,20 @@
 
 namespace mpk {
 
+// Lower a non-negative half-precision threshold hint to min(*p, v) (16-bit CAS: non-negative
+// halves order as their bit patterns).  Hints are read with plain loads by other lanes; an
+// atomic update keeps every read seeing some value that was merged (never a torn or raised one).
+__device__ __forceinline__ void atomic_min_half(__half* p, __half v) {
+    unsigned short* a = reinterpret_cast<unsigned short*>(p);
+    const unsigned short nv = __half_as_ushort(v);
+    unsigned short old = *reinterpret_cast<volatile unsigned short*>(a);
+    while (nv < old) {
+        const unsigned short prev = atomicCAS(a, old, nv);
+        if (prev == old) break;
+        old = prev;
+    }
+}
+
 template <> struct PT<__half2> {
     static __device__ __forceinline__ __half2 vmin(__half2 a, __half2 b) { return __hmin2(a, b); }
     static __device__ __forceinline__ __half2 vmax(__half2 a, __half2 b) { return __hmax2(a, b); }
@@ -434,6 +448,7 @@ mp_diag_h(const MainParams p) {
                     }
                     const bool need_r = __any_sync(FULL, fminf(v[0], v[1]) <= tr);
                     const bool need_c = SELF && __any_sync(FULL, v[0] <= tc[0] || v[1] <= tc[1]);
+                    __syncwarp();   // every lane read the hints before a leader lowers them
                     if (need_r) {
                         float vr = fminf(v[0], v[1]);
 #pragma unroll
@@ -443,7 +458,7 @@ mp_diag_h(const MainParams p) {
                         if (vr < FINF && vr <= tr && lane == __ffs(eqr) - 1) {
                             const int j = (v[0] == vr) ? col0 : col0 + 1;          // lowest column first
                             KeyOps<float>::merge(keys + (size_t)row * d + rk, vr, (unsigned)j);
-                            if (vr < tr) rowv[ixr].t = __float2half_rn(vr);        // exact
+                            if (vr < tr) atomic_min_half(&rowv[ixr].t, __float2half_rn(vr));   // exact
                         }
                     }
                     if (SELF && need_c) {
@@ -460,12 +475,13 @@ mp_diag_h(const MainParams p) {
                                 KeyOps<float>::merge(keys + (size_t)colu * d + rk, vc, (unsigned)row);
                                 if (vc < tc[u]) {
                                     const __half h = __float2half_rn(vc);
-                                    reinterpret_cast<__half*>(&colv[pl * PSC + Gm::scol(colu)].w)[0] = h;
-                                    reinterpret_cast<__half*>(&colv[pl * PSC + Gm::scol(colu - 1)].w)[1] = h;
+                                    atomic_min_half(&reinterpret_cast<__half*>(&colv[pl * PSC + Gm::scol(colu)].w)[0], h);
+                                    atomic_min_half(&reinterpret_cast<__half*>(&colv[pl * PSC + Gm::scol(colu - 1)].w)[1], h);
                                 }
                             }
                         }
                     }
+                    __syncwarp();   // the leaders' hint stores are visible to the next rank's reads
                 }
                 __syncwarp();
             }

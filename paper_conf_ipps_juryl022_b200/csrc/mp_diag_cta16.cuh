@@ -35,6 +35,7 @@
 
 namespace mpk {
 
+
 // Per lane-group-size launch shape (measured on one B200, Mixed self-joins of d = 64 / 128 / 256,
 // n = 32768 / 16384 / 8192): warps per block and steps per staging batch (one block barrier per
 // batch).  d = 64: 4 warps, SB = 2 (61.0 -> 58.9 ms); d = 128: 8 warps (45.7 -> 39.5 ms);
@@ -309,7 +310,7 @@ mp_diag_cta_h(const MainParams p) {
                             const float tr = __half2float(rp->t);
                             if (v <= tr) {
                                 atomicMin(keys + (size_t)row * d + rk, ((K)vb << 32) | (unsigned)col);
-                                if (v < tr) rp->t = hv;
+                                if (v < tr) atomic_min_half(&rp->t, hv);
                             }
                             if (SELF) {
                                 __half* cw = reinterpret_cast<__half*>(&colv[cslot(col) * D + pl].w);
@@ -317,8 +318,8 @@ mp_diag_cta_h(const MainParams p) {
                                 if (v <= tc) {
                                     atomicMin(keys + (size_t)col * d + rk, ((K)vb << 32) | (unsigned)row);
                                     if (v < tc) {
-                                        cw[0] = hv;
-                                        reinterpret_cast<__half*>(&colv[cslot(col - 1) * D + pl].w)[1] = hv;
+                                        atomic_min_half(&cw[0], hv);
+                                        atomic_min_half(&reinterpret_cast<__half*>(&colv[cslot(col - 1) * D + pl].w)[1], hv);
                                     }
                                 }
                             }

@@ -405,13 +405,13 @@ mp_diag_cta64(const MainParams p) {
                         } else {
                             merge_q((size_t)row * d + rk, v, (unsigned)col);
                         }
-                        thr_r = fminf(thr_r, __double2float_ru(v * margin));
+                        atomicMin(reinterpret_cast<unsigned*>(&thr_r), __float_as_uint(__double2float_ru(v * margin)));
                     }
                     if (SELF) {
                         float& thr_c = TA ? TCs[kk] : colv[sc * D + pl].thr;
                         if (v <= (double)thr_c) {
                             merge_q((size_t)col * d + rk, v, (unsigned)row);
-                            thr_c = fminf(thr_c, __double2float_ru(v * margin));
+                            atomicMin(reinterpret_cast<unsigned*>(&thr_c), __float_as_uint(__double2float_ru(v * margin)));
                         }
                     }
                 }

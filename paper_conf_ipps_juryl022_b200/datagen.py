@@ -82,6 +82,37 @@ def random_walk_ab(d: int, n: int, m: int, seed: int, motif: bool = True):
     return np.cumsum(rq, axis=1), np.cumsum(rr, axis=1)
 
 
+PATTERN_NAMES = ["sine", "square", "triangle", "saw", "chirp", "gaussian", "step", "exp-decay"]
+
+
+def pattern_shapes(m: int):
+    """The eight analogue primitive shapes in [-1, 1] over t in [0, 1) (the paper's P0-P7 exist
+    only as a drawing, Fig. 3; SURVEY 8(d) names these analogues)."""
+    t = np.linspace(0.0, 1.0, m)
+    return [np.sin(2 * np.pi * 2 * t), np.sign(np.sin(2 * np.pi * 2 * t)),
+            2 * np.abs(2 * (2 * t % 1) - 1) - 1, 2 * (3 * t % 1) - 1,
+            np.sin(2 * np.pi * (1 + 4 * t) * t), 2 * np.exp(-((t - 0.5) / 0.1) ** 2) - 1,
+            np.where(t < 0.5, -1.0, 1.0), 2 * np.exp(-5 * t) - 1]
+
+
+def embedded_pattern(d: int, n: int, m: int, shape: int, n_occ: int, seed: int, noise: float = 0.25):
+    """(T, starts): N(0, noise^2) noise in d dims with pattern `shape` added at n_occ random,
+    non-overlapping window starts (the paper's stress-test series with randomly located injected
+    repeating patterns, and the embedded-motif recall set-up, L1218-1229)."""
+    L = n + m - 1
+    rng = np.random.default_rng(seed)
+    T = noise * rng.standard_normal((d, L))
+    p = pattern_shapes(m)[shape]
+    starts = []
+    while len(starts) < n_occ:
+        x = int(rng.integers(0, n))
+        if all(abs(x - y) >= 2 * m for y in starts):
+            starts.append(x)
+    for x in starts:
+        T[:, x:x + m] += p
+    return T, sorted(starts)
+
+
 def bounded_patterns(d: int, n: int, m: int, seed: int, n_inject: int = 8) -> np.ndarray:
     """N(0,1) noise with analogue pattern shapes in [-1, 1] (paper-like bounded family)."""
     L = n + m - 1

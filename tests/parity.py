@@ -6,6 +6,7 @@ I:  I_gpu == I_or where the oracle's runner-up gap P2 - P exceeds tol(P); elsewh
     I_gpu whose own oracle value D''_k(i, I_gpu) <= P_or + tol(P) is accepted.
 """
 import math
+import os
 
 import numpy as np
 
@@ -52,7 +53,7 @@ def check(oracle, T, m, P_or, I_or, P2_or, P_gpu, I_gpu, prec, rows=None, Tr=Non
     assert np.array_equal(fin, np.isfinite(Pg)), "finite pattern differs"
     assert np.all(Ig[~fin] == -1) and np.all(I_or[~fin] == -1)
     tol = tol_of(np.where(fin, P_or, 0.0), m, prec, P0_row=np.where(fin[0], P_or[0], np.inf))
-    if cond and prec == "fp32":
+    if cond and prec == "fp32" and not os.environ.get("MP_PARITY_NO_COND"):
         kq = kappa(T, m)
         kr = kq if Tr is None else kappa(Tr, m)
         kj = kr[np.clip(I_or, 0, len(kr) - 1)]
