@@ -349,10 +349,16 @@ def main():
     ap.add_argument("--dry-run", action="store_true",
                     help="functional run of the multi-rank path: one step, no warm-up; the line says "
                          "dry_run and is not a bench value")
+    ap.add_argument("--per-precision", action="store_true",
+                    help="N > 1: also time the other precisions (off by default: C4 FP64 takes minutes per step)")
     args = ap.parse_args()
     args.warmup = 0 if args.dry_run else max(args.warmup, 3)
+    world0 = int(os.environ.get("WORLD_SIZE", "1"))
     if args.dry_run:
         args.steps = 1
+        args.no_per_precision = args.no_context = args.no_per_config = args.no_cpu_baseline = True
+    if world0 > 1 and not args.per_precision:
+        args.no_per_precision = True
     world = int(os.environ.get("WORLD_SIZE", "1"))
     if args.config is None:
         args.config = "C3" if world == 1 else "C4"

@@ -23,18 +23,21 @@
 
 namespace mpk {
 
-// Lower a non-negative half-precision threshold hint to min(*p, v) (16-bit CAS: non-negative
-// halves order as their bit patterns).  Hints are read with plain loads by other lanes; an
-// atomic update keeps every read seeing some value that was merged (never a torn or raised one).
-__device__ __forceinline__ void atomic_min_half(__half* p, __half v) {
-    unsigned short* a = reinterpret_cast<unsigned short*>(p);
-    const unsigned short nv = __half_as_ushort(v);
-    unsigned short old = *reinterpret_cast<volatile unsigned short*>(a);
-    while (nv < old) {
-        const unsigned short prev = atomicCAS(a, old, nv);
-        if (prev == old) break;
-        old = prev;
-    }
+// Lower a non-negative half-precision threshold hint towards v with ONE 32-bit atomicMin on the
+// word holding it (non-negative halves order as their bits; the word's other half is re-used as
+// read).  If the other half was lowered concurrently the atomic may skip this update or restore
+// the other half's older, higher value: a hint can end up higher than the best -- an extra
+// slow-path visit -- but never lower, and never torn.  Plain loads by other lanes always see a
+// value that was merged into the global keys.
+__device__ __forceinline__ void atomic_min_half(__half* p, __half v) {   // p: shared memory
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(p);
+    const unsigned wa = sa & ~3u;
+    const bool hi = (sa & 2u) != 0;
+    unsigned old;
+    asm volatile("ld.volatile.shared.u32 %0, [%1];" : "=r"(old) : "r"(wa) : "memory");
+    const unsigned hv = __half_as_ushort(v);
+    const unsigned nw = hi ? ((hv << 16) | (old & 0xffffu)) : ((old & 0xffff0000u) | hv);
+    asm volatile("red.shared.min.u32 [%0], %1;" ::"r"(wa), "r"(nw) : "memory");
 }
 
 template <> struct PT<__half2> {
