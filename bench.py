@@ -60,6 +60,18 @@ def alu_peak_ops(sm_mhz=None):
     return SM_COUNT * lanes * (sm_mhz or NOMINAL_SM_MHZ) * 1e6
 
 
+def in_memory_bytes(d, n, m, prec, self_join):
+    """Device bytes of the in-memory path's per-position arrays (stats, pair format, seed
+    operands, keys, window-stat scratch) and P / I: what mp_compute_stream bounds."""
+    half = prec in ("fp16", "mixed", "fp16c", "fp16ck")
+    sb = 16 if half else (32 if prec == "fp64" else 16)
+    tb = 8 if prec == "fp64" else (2 if prec in ("fp16", "fp16c") else 4)
+    dp = 1 << (d - 1).bit_length()
+    side = n * d * sb + (n + 1) * d * 16 * half + (n + m - 1) * dp * tb + n * dp * tb + 2 * n * d * (8 if prec == "fp32" else tb)
+    keys = n * d * (16 if prec == "fp64" else 8)
+    return int(side * (1 if self_join else 2) + keys + 16 * d * n)
+
+
 def batcher_ce(N: int) -> int:
     """Comparators of Batcher's odd-even merge sort network on N inputs (as sort_net builds it)."""
     c = 0
@@ -181,7 +193,7 @@ def alu_ops_mode(d: int, self_join: bool, prec: str) -> float:
     the FP32 filter: same sort, scan and compares) as alu_ops_per_cell_dim; FP16 / Mixed pack two
     cells in a half2, so each HMNMX2 / HSETP2 serves two cell*dims."""
     ops = alu_ops_per_cell_dim(d, self_join)
-    return ops / 2.0 if prec in ("fp16", "mixed", "fp16c") else ops
+    return ops / 2.0 if prec in ("fp16", "mixed", "fp16c", "fp16ck") else ops
 
 
 _PROBE_CACHE = {}
@@ -349,6 +361,9 @@ def main():
     ap.add_argument("--dry-run", action="store_true",
                     help="functional run of the multi-rank path: one step, no warm-up; the line says "
                          "dry_run and is not a bench value")
+    ap.add_argument("--no-stream", action="store_true", help="skip the beyond-memory streaming leg")
+    ap.add_argument("--stream-bytes", type=int, default=512 << 20,
+                    help="device budget of the streaming leg (mp_compute_stream)")
     ap.add_argument("--per-precision", action="store_true",
                     help="N > 1: also time the other precisions (off by default: C4 FP64 takes minutes per step)")
     args = ap.parse_args()
@@ -357,6 +372,7 @@ def main():
     if args.dry_run:
         args.steps = 1
         args.no_per_precision = args.no_context = args.no_per_config = args.no_cpu_baseline = True
+        args.no_stream = True
     if world0 > 1 and not args.per_precision:
         args.no_per_precision = True
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -533,6 +549,25 @@ def main():
                "h2d_bytes_per_step": d * L * 8 * (1 if self_join else 2), "d2h_bytes_per_step": 2 * d * n * 8,
                "ms_per_step": statistics.mean(ts) * 1e3}
 
+    # beyond-memory streaming (mp_compute_stream, NEXT-4): the same job with a device budget far
+    # below the in-memory footprint; host T in, host P / I out (timed like e2e), checked bit for
+    # bit against the in-memory result of the e2e leg
+    stream = None
+    if world == 1 and not args.no_stream:
+        Ps = (np.empty((d, n)), np.empty((d, n), dtype=np.int64))
+        t0 = time.perf_counter()
+        ctx.compute_stream(Th, m, args.precision, e, Tr=Trh, device_bytes=args.stream_bytes, out=Ps)
+        dt = time.perf_counter() - t0
+        R, Wb, peak, nl = ctx.last_stream_info()
+        skms, _ = ctx.last_timing()
+        stream = {"value": dn2 / dt, "unit": UNIT, "ms": dt * 1e3, "main_kernel_ms": skms,
+                  "device_bytes": args.stream_bytes, "peak_mapped_bytes": peak, "rows_per_chunk": R,
+                  "diagonals_per_band": Wb, "launches": nl,
+                  "in_memory_device_bytes": in_memory_bytes(d, n, m, args.precision, self_join),
+                  "bit_identical_to_in_memory": bool(np.array_equal(Ps[0], outs[0]) and np.array_equal(Ps[1], outs[1])),
+                  "vs_e2e": (dn2 / dt) / e2e["value"] if e2e else None}
+        del Ps
+
     if rank == 0:
         peaks, src = load_peaks()
         # roofline of the dominant kernel: algorithmic ops of the cells THIS launch computed (rank
@@ -545,7 +580,7 @@ def main():
         lanes, lsrc = alu_lanes()
         peak_tops = peak_ops / 1e12
         achieved = ops / (kms * 1e-3) / 1e12 if kms > 0 else None
-        kname = {"fp32": "mp_diag_cta" if d > 32 else "mp_diag", "fp64": "mp_diag_cta64" if d > 32 else "mp_diag64f"}
+        kname = {"fp32": "mp_diag_ctab" if d > 32 else "mp_diag", "fp64": "mp_diag_cta64" if d > 32 else "mp_diag64f"}
         roof = {"bound": "alu", "achieved": achieved, "peak": peak_tops, "unit": "Tops/s",
                 "frac": achieved / peak_tops if achieved else None,
                 "traffic": load_traffic(args.config, args.precision),
@@ -553,7 +588,7 @@ def main():
                 "ops_per_cell_dim": alu_ops_mode(d, self_join, args.precision),
                 "ops_basis": "SURVEY 8(d): clamp 1 + 2 CE(d_pad)/d + 3 per profile side",
                 "frac_filtered_ops": (alu_ops_filtered(d, self_join) * band_cells * d / (kms * 1e-3) / 1e12 / peak_tops
-                                      / (2.0 if args.precision in ("fp16", "mixed", "fp16c") else 1.0)) if kms > 0 else None,
+                                      / (2.0 if args.precision in ("fp16", "mixed", "fp16c", "fp16ck") else 1.0)) if kms > 0 else None,
                 "computed_cell_dims": band_cells * d,
                 "peak_basis": f"{SM_COUNT} SM x {lanes:.2f} FMNMX lanes/SM/clk ({lsrc}: scripts/pipe_peaks.cu -> "
                               f"profiles/r1_pipe_peaks.json; MEASURED_PEAKS {src} has no ALU figure) x {run_mhz:.0f} MHz "
@@ -569,7 +604,8 @@ def main():
                 "data": "synthetic", "config": config_json(args, cfg), "roofline": roof, "cpu_baseline": cpu,
                 "e2e": e2e, "gpu_launches": launches_per_step(args.precision, self_join) * args.steps,
                 "clocks": clocks, "per_precision": per_prec, "context": context,
-                "per_config_band": per_cfg or None, "computed_cells_per_s": cells * d / (ms * 1e-3)}
+                "per_config_band": per_cfg or None, "computed_cells_per_s": cells * d / (ms * 1e-3),
+                "stream": stream}
         if merge_check is not None:
             line["merge_check"] = merge_check
         if args.dry_run:

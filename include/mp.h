@@ -50,9 +50,13 @@ typedef enum {
     MP_FP64 = 0,   /* precalculation FP64, main loop FP64           (L426-428, L764-766) */
     MP_FP32 = 1,   /* precalculation FP32, main loop FP32           (L430-432, L771-772) */
     MP_FP16 = 2,   /* precalculation FP16, main loop FP16           (L434-436, L773-776) */
-    MP_MIXED = 3,  /* precalculation FP32, main loop FP16           (L438-440, L777-785) */
-    MP_FP16C = 4   /* precalculation FP16 with Kahan-compensated sums, main loop FP16
-                      (Fig. 1 "FP16 with compensator" L442-444, L786-798; G17) */
+    MP_MIXED = 3,  /* precalculation FP32 (plain sums), main loop FP16 (L438-440, L777-785) */
+    MP_FP16C = 4,  /* precalculation FP16 with Kahan-compensated sums, main loop FP16
+                      (Fig. 1 "FP16 with compensator" L442-444; G17, Fig. 1 reading) */
+    MP_FP16CK = 5  /* FP16C, the text's reading: precalculation (window statistics and seeds) in
+                      FP32 arithmetic with Kahan-compensated sums, main loop FP16 (L786-798
+                      "higher precision mode in precalculation ... Kahan's compensated
+                      summation"; G17, text reading).  Re-seed interval of MIXED. */
 } mp_precision;
 
 #define MP_MAX_D 1024
@@ -61,7 +65,8 @@ typedef struct mp_ctx mp_ctx;   /* opaque */
 
 typedef struct {
     int device;             /* CUDA device ordinal this context drives (one process per GPU) */
-    int64_t reseed_h[4];    /* re-seed interval H (rows) for FP64, FP32, FP16 (also FP16C), MIXED;
+    int64_t reseed_h[4];    /* re-seed interval H (rows) for FP64, FP32, FP16 (also FP16C), MIXED
+                               (also FP16CK);
                                0 -> default (R2); rounded up to a multiple of 8 (re-seeds
                                fall on staging-batch starts); < 0 or > 2^30 -> MP_ERR_INVALID */
 } mp_config;
@@ -142,6 +147,38 @@ mp_status mp_plan_diagonals(int64_t d, int64_t n, int64_t m, mp_precision prec, 
 /* Kernel timing of the last mp_compute* / mp_partial_device call on ctx (ms, CUDA
  * events around the main diagonal kernel only) and its launch count. */
 mp_status mp_last_timing(const mp_ctx* ctx, double* main_kernel_ms, int64_t* launches);
+
+/*
+ * Beyond-memory streaming (the tiling "decouples the size
+ * of the distance matrix" from "the limited device memory", and L2432-2433).
+ *
+ * mp_compute_stream: the same result as mp_compute -- bit-identical P and I for every precision
+ *   -- computed with at most about `device_bytes` of device memory for the per-position arrays
+ *   (statistics, seed operands, merge keys), independent of n.  T, Tr, P, I and the running merge
+ *   keys stay in host memory (the library allocates a pinned key store of n*d*8 bytes, n*d*16
+ *   for FP64, for the duration of the call).  The tile plan is cut into row chunks of R rows
+ *   (a multiple of the tile height) times diagonal bands of Wb diagonals; per step the device
+ *   holds one row window and one column window (CUDA virtual memory: full-size address
+ *   reservations, physical memory mapped for the windows only), computes the window statistics
+ *   from a T slice, restores / saves the keys of the windows, and finalizes rows [i0, i1) when
+ *   their chunk is done.  Arguments as mp_compute; device_bytes > 0.  Errors: MP_ERR_NOMEM when
+ *   device_bytes cannot hold one row segment of the plan; MP_ERR_UNSUPPORTED when the driver
+ *   lacks the virtual-memory entry points.  Scratch cached on ctx by other calls is not counted.
+ *   Testing knobs: the environment variables MP_STREAM_ROWS / MP_STREAM_DIAGS override R / Wb
+ *   (rounded up to the tile height / block width) so small inputs exercise many chunks.
+ * mp_plan_stream: the chunk geometry (rows per chunk R, diagonals per band Wb) mp_compute_stream
+ *   chooses for a budget and an allocation granularity (bytes; the device's is 2 MiB).  Host
+ *   only, no GPU needed.  MP_ERR_NOMEM as above.
+ * mp_last_stream_info: R, Wb, the peak physically mapped bytes and the number of fused-kernel
+ *   launches of the last mp_compute_stream on ctx (mp_last_timing gives the summed kernel time).
+ */
+mp_status mp_compute_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, int64_t n, int64_t m,
+                            mp_precision prec, int64_t exclusion, int64_t device_bytes, double* P, int64_t* I);
+mp_status mp_plan_stream(int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion, int self_join,
+                         int64_t device_bytes, int64_t granularity, int64_t* rows_per_chunk,
+                         int64_t* diagonals_per_band);
+mp_status mp_last_stream_info(const mp_ctx* ctx, int64_t* rows_per_chunk, int64_t* diagonals_per_band,
+                              int64_t* peak_device_bytes, int64_t* launches);
 
 /*
  * Stage self-tests (per-stage unit tests of SURVEY 4; tests/test_gpu_stages.py).  They run ONE

@@ -56,12 +56,35 @@ def _stale():
         return f.read().strip() != _digest()
 
 
+def _obj_digest(src, cmd):
+    """Content hash of one object's inputs: the command, the source and every header it can
+    include (host sources: include/ and the internal header; CUDA sources: all csrc headers)."""
+    h = hashlib.sha256()
+    h.update(" ".join(cmd).encode())
+    inc = os.path.join(HERE, "..", "include")
+    hdrs = [os.path.join(inc, x) for x in os.listdir(inc)]
+    if src.endswith(".cpp"):
+        hdrs.append(os.path.join(CSRC, "mp_internal.h"))
+    else:
+        hdrs += [os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith((".cuh", ".h"))]
+    for f in [src] + sorted(hdrs):
+        with open(f, "rb") as fh:
+            h.update(fh.read())
+    return h.hexdigest()
+
+
 def _compile(src):
     obj = os.path.join(OBJDIR, os.path.basename(src) + ".o")
     cmd = [NVCC] + ARCH + FLAGS + ["-c", src, "-o", obj]
     if os.environ.get("MP_PTXAS_V"):
         cmd += ["-Xptxas", "-v"]
+    dg = _obj_digest(src, cmd)
+    stamp = obj + ".sha256"
+    if os.path.exists(obj) and os.path.exists(stamp) and open(stamp).read().strip() == dg:
+        return obj   # unchanged inputs: reuse the object (incremental rebuild)
     subprocess.check_call(cmd)
+    with open(stamp, "w") as f:
+        f.write(dg + "\n")
     return obj
 
 

@@ -9,18 +9,20 @@
 #include "../../include/mp.h"
 #include "mp_internal.h"
 
+#include <cuda.h>           // driver-API types only (VMM entry points are fetched at run time)
 #include <cuda_runtime.h>
 
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
 
 namespace {
 
-constexpr int64_t kDefaultH[5] = {4096, 1024, 256, 256, 256};  // FP64, FP32, FP16, MIXED, FP16C (upper bounds)
+constexpr int64_t kDefaultH[6] = {4096, 1024, 256, 256, 256, 256};  // FP64, FP32, FP16, MIXED, FP16C, FP16CK (upper bounds)
 
 // Default re-seed interval H (= tile height, the paper's tiling lever against error growth,
 // PAPER.md:L700-703).  The recurrence error grows with H relative to the window energy, which
@@ -42,7 +44,7 @@ struct mp_ctx {
     int device = 0;
     int nsm = 148;
     cudaStream_t stream = nullptr;
-    int64_t H[5] = {0, 0, 0, 0, 0};
+    int64_t H[6] = {0, 0, 0, 0, 0, 0};
     std::string err;
     // cached scratch
     Buf dT, dTr, st_q, st_r, tw_q, tw_r, mu_q, mu_r, mup_q, mup_r, nrm, keys, ext, seg, counter, dP, dI, flag;
@@ -51,6 +53,9 @@ struct mp_ctx {
     int* hflag = nullptr;   // pinned read-back of the non-finite flag
     double last_ms = 0.0;
     int64_t last_launches = 0;
+    // last mp_compute_stream: chunk geometry and peak physically mapped device bytes
+    int64_t stream_R = 0, stream_Wb = 0, stream_peak = 0, stream_launches = 0;
+    bool stream_timed = false;   // last_ms is the sum over the streamed launches
 };
 
 namespace {
@@ -89,6 +94,11 @@ void release(Buf& b) {
 }
 
 size_t elt_bytes(int prec) { return prec == MP_FP64 ? 8 : 4; }
+
+// precompute over the whole series (every position resident)
+void full_window(mpk::PreParams& pp, int64_t n, int64_t L) {
+    pp.w0 = 0; pp.w1 = n; pp.T_off = 0; pp.T_ld = L; pp.s_off = 0; pp.s_end = n; pp.s_ld = n;
+}
 
 // ---------------------------------------------------------------- tile plan
 struct Plan {
@@ -160,9 +170,90 @@ mp_status validate(mp_ctx* ctx, const void* T, int64_t d, int64_t n, int64_t m, 
     if (m < 2) return fail(ctx, MP_ERR_INVALID, "m must be >= 2");
     if (n >= (int64_t(1) << 31) - 1) return fail(ctx, MP_ERR_INVALID, "n must be < 2^31");
     if (m > (int64_t(1) << 20)) return fail(ctx, MP_ERR_INVALID, "m too large");
-    if (prec < 0 || prec > 4) return fail(ctx, MP_ERR_INVALID, "unknown precision");
+    if (prec < 0 || prec > 5) return fail(ctx, MP_ERR_INVALID, "unknown precision");
     if (prec == MP_FP64 && d > 512) return fail(ctx, MP_ERR_UNSUPPORTED, "FP64 supports d <= 512");
     return MP_OK;
+}
+
+// Launch the fused kernel over the tiles of diagonal blocks [B0, B1) of plan pl restricted to the
+// row segments [q0, q1) (a whole band: q0 = 0, q1 = nq).  The band's blocks are renumbered from 0
+// (delta_lo = the band's first diagonal), so every tile -- diagonal block x row segment, seeds at
+// the segment start and at the fixed re-seed rows -- is the same computation as in the full plan:
+// results do not depend on how the plan is cut into launches (ranks, streamed chunks).
+// mp carries the data pointers and n, d, m, H; the tile fields are filled here.
+mp_status enqueue_tiles(mp_ctx* ctx, cudaStream_t s, int prec, bool self, mpk::MainParams mp, const Plan& pl,
+                        int64_t B0, int64_t B1, int64_t q0, int64_t q1, bool timed) {
+    const int64_t n = mp.n, HT = pl.H, NC = pl.nc, nb = B1 - B0;
+    if (nb <= 0 || q1 <= q0) return MP_OK;
+    const int64_t dlo = pl.dlo + B0 * NC, dhi = std::min<int64_t>(pl.dlo + B1 * NC - 1, pl.dhi);
+    const int64_t nq = std::max<int64_t>(1, (n + HT - 1) / HT);
+    // segments [qlo(b), qhi(b)) of band block b inside [q0, q1); both are non-increasing in b
+    auto qlo = [&](int64_t b) {
+        const int64_t d1 = std::min(dlo + b * NC + NC - 1, dhi);
+        return std::max<int64_t>(q0, std::max<int64_t>(0, -d1) / HT);
+    };
+    auto qhi = [&](int64_t b) {
+        const int64_t d0 = dlo + b * NC;
+        return std::min<int64_t>(q1, (std::min<int64_t>(n, n - std::max<int64_t>(d0, 0)) + HT - 1) / HT);
+    };
+    auto first_b = [&](auto pred) {  // first b in [0, nb) with pred(b) (monotone), else nb
+        int64_t lo = 0, hi = nb;
+        while (lo < hi) {
+            const int64_t mid = (lo + hi) / 2;
+            if (pred(mid)) hi = mid; else lo = mid + 1;
+        }
+        return lo;
+    };
+    // [q_prefix (nq + 1) | q_block0 (nq) | seg_prefix (nb + 1)]
+    std::vector<long long> tab(2 * nq + 1 + nb + 1);
+    tab[0] = 0;
+    for (int64_t q = 0; q < nq; ++q) {  // segment-major order (warp-tile kernels)
+        const int64_t bs = first_b([&](int64_t b) { return qlo(b) <= q; });
+        const int64_t be = first_b([&](int64_t b) { return qhi(b) <= q; });
+        tab[q + 1] = tab[q] + std::max<int64_t>(0, be - bs);
+        tab[nq + 1 + q] = bs;
+    }
+    long long* segp = tab.data() + 2 * nq + 1;   // block-major order (block-cooperative kernels)
+    segp[0] = 0;
+    for (int64_t b = 0; b < nb; ++b) segp[b + 1] = segp[b] + std::max<int64_t>(0, qhi(b) - qlo(b));
+    const long long total = segp[nb];
+    if (tab[nq] != total) return fail(ctx, MP_ERR_INVALID, "internal: tile plan mismatch");
+    if (total == 0) return MP_OK;
+    MP_CUDA(ctx, ensure(ctx->seg, tab.size() * sizeof(long long)));
+    MP_CUDA(ctx, cudaMemcpyAsync(ctx->seg.p, tab.data(), tab.size() * sizeof(long long), cudaMemcpyHostToDevice, s));
+    MP_CUDA(ctx, ensure(ctx->counter, sizeof(unsigned long long)));
+    MP_CUDA(ctx, cudaMemsetAsync(ctx->counter.p, 0, sizeof(unsigned long long), s));
+    const mpk::Variant var = mpk::pick_variant(prec, mp.d);
+    mp.order = var.cta ? 0 : 1;   // decode_tile (mp_diag.cuh) says why
+    mp.q_prefix = (const long long*)ctx->seg.p;
+    mp.q_block0 = (const long long*)ctx->seg.p + nq + 1;
+    mp.nq = nq;
+    mp.seg_prefix = (const long long*)ctx->seg.p + 2 * nq + 1;
+    mp.nb = nb;
+    mp.t_begin = 0;
+    mp.t_count = total;
+    mp.counter = (unsigned long long*)ctx->counter.p;
+    mp.HT = pl.H;
+    mp.delta_lo = dlo; mp.delta_hi = dhi;
+    mp.q_lo = q0;
+    const int bps = std::max(1, mpk::main_blocks_per_sm(prec, mp.d, self));
+    long long grid = (long long)ctx->nsm * bps;
+    const int wpb = std::max(1, mpk::variant_warps_per_block(prec, mp.d, self));
+    grid = std::min<long long>(grid, (total + wpb - 1) / wpb);
+    grid = std::max<long long>(grid, 1);
+    if (timed) MP_CUDA(ctx, cudaEventRecord(ctx->ev0, s));
+    MP_CUDA(ctx, mpk::launch_main(prec, self, mp, (int)grid, s));
+    if (timed) MP_CUDA(ctx, cudaEventRecord(ctx->ev1, s));
+    ctx->last_launches += 1;
+    return MP_OK;
+}
+
+// Re-seed interval of a run: the context's (mp_config.reseed_h) or the default, rounded up to a
+// multiple of 8 (every kernel steps in batches of 1, 2 or 4 rows, so every re-seed row
+// i = 0 mod H is a batch start in every kernel variant; include/mp.h, mp_config.reseed_h).
+int64_t reseed_interval(const mp_ctx* ctx, int prec, int64_t m) {
+    const int64_t H = ctx->H[prec] > 0 ? ctx->H[prec] : default_h(prec, m);
+    return std::min<int64_t>((H + 7) / 8 * 8, int64_t(1) << 30);
 }
 
 // Device pipeline: keys for band (rank, world) of the tile plan, internal key format.
@@ -174,8 +265,8 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     // re-seeds happen at staging-batch starts (every kernel steps in batches of 1, 2 or 4 rows),
     // so the interval is rounded up to a multiple of 8: then every re-seed row i = 0 mod H is a
     // batch start in every kernel variant (include/mp.h, mp_config.reseed_h)
-    int64_t H = ctx->H[prec] > 0 ? ctx->H[prec] : default_h(prec, m);
-    H = std::min<int64_t>((H + 7) / 8 * 8, int64_t(1) << 30);
+    const int64_t H = reseed_interval(ctx, prec, m);
+    ctx->stream_timed = false;
     if (self && excl < 0) excl = (m + 3) / 4;
 
     // flag non-finite inputs (reading G23).  The flag is read back after the whole pipeline is
@@ -188,7 +279,7 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     if (!self) MP_CUDA(ctx, mpk::launch_check_finite(dTr, d * L, (int*)ctx->flag.p, s));
 
     // precalculation (Pseudocode 1 line 2)
-    const bool half = prec == MP_FP16 || prec == MP_MIXED || prec == MP_FP16C;
+    const bool half = prec == MP_FP16 || prec == MP_MIXED || prec == MP_FP16C || prec == MP_FP16CK;
     const size_t sb = half ? 16 : 4 * eb;                                   // stats entry bytes
     const size_t tb = prec == MP_FP64 ? 8 : ((prec == MP_FP16 || prec == MP_FP16C) ? 2 : 4);  // precalc value bytes
     const size_t tbs = prec == MP_FP32 ? 8 : tb;  // window stats scratch (FP32 mode: FP64 precalc, reading R1')
@@ -196,6 +287,7 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     const int Dp = var.DL * var.G;
     mpk::PreParams pp{};
     pp.n = n; pp.d = (int)d; pp.m = (int)m; pp.Dp = Dp;
+    full_window(pp, n, L);
     if (var.ctab) { pp.pm_G = var.G; pp.pm_DL = var.DL; }
     MP_CUDA(ctx, ensure(ctx->nrm, (size_t)n * d * tbs));
     pp.nrm32 = (float*)ctx->nrm.p; pp.nrm64 = (double*)ctx->nrm.p;
@@ -230,75 +322,19 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     ctx->last_ms = 0.0;
     if (pl.nb > 0) {
         std::vector<int64_t> bb = band_blocks(pl, world);
-        const long long t_begin = pl.seg[bb[rank]], t_end = pl.seg[bb[rank + 1]];
-        // segment-major tile order over the band's blocks [B0, B1): for row segment q the
-        // blocks with a tile in it are contiguous, [first b with qlo_b <= q, first b with
-        // qhi_b <= q), because a block's first and last rows never increase with b
-        const int64_t B0 = bb[rank], B1 = bb[rank + 1], HT = pl.H;
-        const int64_t nq = std::max<int64_t>(1, (n + HT - 1) / HT);
-        auto qlo = [&](int64_t b) {
-            const int64_t d1 = std::min(pl.dlo + b * pl.nc + pl.nc - 1, pl.dhi);
-            return std::max<int64_t>(0, -d1) / HT;
-        };
-        auto qhi = [&](int64_t b) {
-            const int64_t d0 = pl.dlo + b * pl.nc;
-            return (std::min<int64_t>(n, n - std::max<int64_t>(d0, 0)) + HT - 1) / HT;
-        };
-        auto first_b = [&](auto pred) {  // first b in [B0, B1) with pred(b) (monotone), else B1
-            int64_t lo = B0, hi = B1;
-            while (lo < hi) {
-                const int64_t mid = (lo + hi) / 2;
-                if (pred(mid)) hi = mid; else lo = mid + 1;
-            }
-            return lo;
-        };
-        std::vector<long long> qtab(2 * nq + 1);  // [q_prefix (nq + 1) | q_block0 (nq) | ...]
-        qtab[0] = 0;
-        for (int64_t q = 0; q < nq; ++q) {
-            const int64_t bs = first_b([&](int64_t b) { return qlo(b) <= q; });
-            const int64_t be = first_b([&](int64_t b) { return qhi(b) <= q; });
-            qtab[q + 1] = qtab[q] + std::max<int64_t>(0, be - bs);
-            qtab[nq + 1 + q] = bs;
-        }
-        if (qtab[nq] != t_end - t_begin) return fail(ctx, MP_ERR_INVALID, "internal: tile plan mismatch");
-        qtab.insert(qtab.end(), pl.seg.begin(), pl.seg.end());  // [.. | seg_prefix (nb + 1)]
-        MP_CUDA(ctx, ensure(ctx->seg, qtab.size() * sizeof(long long)));
-        MP_CUDA(ctx, cudaMemcpyAsync(ctx->seg.p, qtab.data(), qtab.size() * sizeof(long long),
-                                     cudaMemcpyHostToDevice, s));
-        MP_CUDA(ctx, ensure(ctx->counter, sizeof(unsigned long long)));
-        MP_CUDA(ctx, cudaMemsetAsync(ctx->counter.p, 0, sizeof(unsigned long long), s));
-        if (t_end > t_begin) {
-            mpk::MainParams mp{};
-            mp.st_q = ctx->st_q.p;
-            mp.st_r = self ? ctx->st_q.p : ctx->st_r.p;
-            if (half) mp.st_r = self ? ctx->stp_q.p : ctx->stp_r.p;   // columns: pair format
-            mp.tw_q = ctx->tw_q.p;
-            mp.tw_r = self ? ctx->tw_q.p : ctx->tw_r.p;
-            mp.mu_q = ctx->mup_q.p;
-            mp.mu_r = self ? ctx->mup_q.p : ctx->mup_r.p;
-            mp.keys = ctx->keys.p;
-            mp.order = var.cta ? 0 : 1;   // decode_tile (mp_diag.cuh) says why
-            mp.q_prefix = (const long long*)ctx->seg.p;
-            mp.q_block0 = (const long long*)ctx->seg.p + nq + 1;
-            mp.nq = nq;
-            mp.seg_prefix = (const long long*)ctx->seg.p + 2 * nq + 1;
-            mp.nb = pl.nb;
-            mp.t_begin = t_begin;
-            mp.t_count = t_end - t_begin;
-            mp.counter = (unsigned long long*)ctx->counter.p;
-            mp.n = n; mp.d = (int)d; mp.m = (int)m; mp.H = (int)H; mp.HT = pl.H;
-            mp.delta_lo = pl.dlo; mp.delta_hi = pl.dhi;
-            const int bps = std::max(1, mpk::main_blocks_per_sm(prec, (int)d, self));
-            const long long want_warps = mp.t_count;
-            long long grid = (long long)ctx->nsm * bps;
-            const int wpb = std::max(1, mpk::variant_warps_per_block(prec, (int)d, self));
-            grid = std::min<long long>(grid, (want_warps + wpb - 1) / wpb);
-            grid = std::max<long long>(grid, 1);
-            MP_CUDA(ctx, cudaEventRecord(ctx->ev0, s));
-            MP_CUDA(ctx, mpk::launch_main(prec, self, mp, (int)grid, s));
-            MP_CUDA(ctx, cudaEventRecord(ctx->ev1, s));
-            ctx->last_launches = 1;
-        }
+        mpk::MainParams mp{};
+        mp.st_q = ctx->st_q.p;
+        mp.st_r = self ? ctx->st_q.p : ctx->st_r.p;
+        if (half) mp.st_r = self ? ctx->stp_q.p : ctx->stp_r.p;   // columns: pair format
+        mp.tw_q = ctx->tw_q.p;
+        mp.tw_r = self ? ctx->tw_q.p : ctx->tw_r.p;
+        mp.mu_q = ctx->mup_q.p;
+        mp.mu_r = self ? ctx->mup_q.p : ctx->mup_r.p;
+        mp.keys = ctx->keys.p;
+        mp.n = n; mp.d = (int)d; mp.m = (int)m; mp.H = (int)H;
+        mp.seed_kahan = prec == MP_FP16CK ? 1 : 0;
+        const int64_t nq = std::max<int64_t>(1, (n + pl.H - 1) / pl.H);
+        return enqueue_tiles(ctx, s, prec, self, mp, pl, bb[rank], bb[rank + 1], 0, nq, true);
     }
     return MP_OK;
 }
@@ -311,6 +347,436 @@ mp_status finish_partial(mp_ctx* ctx, cudaStream_t s) {
     MP_CUDA(ctx, cudaStreamSynchronize(s));
     if (*ctx->hflag) return fail(ctx, MP_ERR_INVALID, "non-finite input");
     return MP_OK;
+}
+
+
+// ---------------------------------------------------------------- beyond-memory streaming (NEXT-4)
+// PAPER.md:L693-699 (the tiling "decouples the size of the distance matrix ... despite the
+// limited device memory") and L2432-2433; SURVEY 8(f) NEXT-4.  The host keeps T, Tr and the
+// running merge keys; the device holds, per step, the statistics / seed operands / keys of one
+// row window [i0, i1) and one column window (the columns of a diagonal band over those rows).
+// Every device array keeps its absolute-position layout inside a virtual-address reservation of
+// the full size (CUDA VMM): only the granules of the current windows are backed by physical
+// memory, so the fused kernels run unchanged, and a position outside the windows would fault.
+
+typedef CUresult (*PF_memCreate)(CUmemGenericAllocationHandle*, size_t, const CUmemAllocationProp*, unsigned long long);
+typedef CUresult (*PF_memRelease)(CUmemGenericAllocationHandle);
+typedef CUresult (*PF_addrReserve)(CUdeviceptr*, size_t, size_t, CUdeviceptr, unsigned long long);
+typedef CUresult (*PF_addrFree)(CUdeviceptr, size_t);
+typedef CUresult (*PF_memMap)(CUdeviceptr, size_t, size_t, CUmemGenericAllocationHandle, unsigned long long);
+typedef CUresult (*PF_memUnmap)(CUdeviceptr, size_t);
+typedef CUresult (*PF_memSetAccess)(CUdeviceptr, size_t, const CUmemAccessDesc*, size_t);
+typedef CUresult (*PF_memGran)(size_t*, const CUmemAllocationProp*, CUmemAllocationGranularity_flags);
+
+struct VArr {                                      // one virtual array
+    CUdeviceptr base = 0;
+    size_t bytes = 0;                              // reserved (a multiple of the granularity)
+    std::vector<CUmemGenericAllocationHandle> h;   // per granule, 0 = unmapped
+    std::vector<char> saved;                       // keys: the granule's bytes live in the host store
+    void* ptr() const { return (void*)base; }
+};
+
+struct Vmm {
+    PF_memCreate create = nullptr; PF_memRelease release = nullptr; PF_addrReserve reserve = nullptr;
+    PF_addrFree afree = nullptr; PF_memMap map = nullptr; PF_memUnmap unmap = nullptr;
+    PF_memSetAccess access = nullptr; PF_memGran granularity = nullptr;
+    CUmemAllocationProp prop{};
+    CUmemAccessDesc acc{};
+    size_t gran = 0, mapped = 0, peak = 0;
+    std::vector<CUmemGenericAllocationHandle> pool;   // unmapped physical granules, reused
+    std::vector<VArr*> arrs;
+
+    std::string load(int dev) {
+        auto get = [](const char* name, void** fp) {
+            cudaDriverEntryPointQueryResult q;
+            return cudaGetDriverEntryPoint(name, fp, cudaEnableDefault, &q) == cudaSuccess &&
+                   q == cudaDriverEntryPointSuccess && *fp != nullptr;
+        };
+        if (!get("cuMemCreate", (void**)&create) || !get("cuMemRelease", (void**)&release) ||
+            !get("cuMemAddressReserve", (void**)&reserve) || !get("cuMemAddressFree", (void**)&afree) ||
+            !get("cuMemMap", (void**)&map) || !get("cuMemUnmap", (void**)&unmap) ||
+            !get("cuMemSetAccess", (void**)&access) || !get("cuMemGetAllocationGranularity", (void**)&granularity))
+            return "CUDA driver VMM entry points unavailable";
+        prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+        prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+        prop.location.id = dev;
+        acc.location = prop.location;
+        acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+        if (granularity(&gran, &prop, CU_MEM_ALLOC_GRANULARITY_RECOMMENDED) != CUDA_SUCCESS || gran == 0)
+            return "cuMemGetAllocationGranularity failed";
+        return "";
+    }
+    CUresult reserve_arr(VArr& a, size_t bytes) {
+        a.bytes = std::max<size_t>(gran, (bytes + gran - 1) / gran * gran);
+        CUresult r = reserve(&a.base, a.bytes, gran, 0, 0);
+        if (r != CUDA_SUCCESS) { a.base = 0; return r; }
+        a.h.assign(a.bytes / gran, 0);
+        a.saved.assign(a.bytes / gran, 0);
+        arrs.push_back(&a);
+        return CUDA_SUCCESS;
+    }
+    CUresult map_g(VArr& a, size_t g) {
+        CUmemGenericAllocationHandle hd = 0;
+        if (!pool.empty()) { hd = pool.back(); pool.pop_back(); }
+        else { CUresult r = create(&hd, gran, &prop, 0); if (r != CUDA_SUCCESS) return r; }
+        CUresult r = map(a.base + g * gran, gran, 0, hd, 0);
+        if (r == CUDA_SUCCESS) r = access(a.base + g * gran, gran, &acc, 1);
+        if (r != CUDA_SUCCESS) { pool.push_back(hd); return r; }
+        a.h[g] = hd;
+        mapped += gran;
+        peak = std::max(peak, mapped);
+        return CUDA_SUCCESS;
+    }
+    CUresult unmap_g(VArr& a, size_t g) {
+        CUresult r = unmap(a.base + g * gran, gran);
+        pool.push_back(a.h[g]);
+        a.h[g] = 0;
+        mapped -= gran;
+        return r;
+    }
+    void destroy() {
+        for (VArr* a : arrs) {
+            for (size_t g = 0; g < a->h.size(); ++g) if (a->h[g]) unmap_g(*a, g);
+            if (a->base) afree(a->base, a->bytes);
+            a->base = 0;
+        }
+        arrs.clear();
+        for (auto hd : pool) release(hd);
+        pool.clear();
+    }
+};
+
+using Ivl = std::pair<int64_t, int64_t>;   // position interval [first, second)
+
+std::vector<Ivl> merge_ivls(std::vector<Ivl> v) {
+    std::vector<Ivl> o;
+    std::sort(v.begin(), v.end());
+    for (const Ivl& x : v) {
+        if (x.first >= x.second) continue;
+        if (!o.empty() && x.first <= o.back().second) o.back().second = std::max(o.back().second, x.second);
+        else o.push_back(x);
+    }
+    return o;
+}
+std::vector<Ivl> minus_ivls(const std::vector<Ivl>& a, const std::vector<Ivl>& b) {  // a \ b (both merged)
+    std::vector<Ivl> o;
+    for (Ivl x : a) {
+        int64_t lo = x.first;
+        for (const Ivl& y : b) {
+            if (y.second <= lo || y.first >= x.second) continue;
+            if (y.first > lo) o.push_back({lo, y.first});
+            lo = std::max(lo, y.second);
+        }
+        if (lo < x.second) o.push_back({lo, x.second});
+    }
+    return o;
+}
+
+// Chunk geometry of a streamed run: rows per chunk R (a multiple of the tile height) and
+// diagonals per band Wb (a multiple of the block width, Wb ~ 2R), the largest that fit the
+// device budget (bytes per resident position x window sizes + fixed granule margins).
+struct StreamGeo {
+    int64_t R = 0, Wb = 0, HT = 0, NC = 0;
+    double per_R = 0, fixed = 0;
+    size_t sb = 0, tb = 0, tbs = 0, kb = 0;
+    int Dp = 0;
+    bool half = false;
+};
+mp_status plan_stream(mp_ctx* ctx, int64_t d, int64_t n, int64_t m, int prec, int64_t excl, bool self,
+                      int64_t budget, size_t gran, const Plan& pl, StreamGeo& g) {
+    const mpk::Variant var = mpk::pick_variant(prec, (int)d);
+    g.half = prec == MP_FP16 || prec == MP_MIXED || prec == MP_FP16C || prec == MP_FP16CK;
+    g.sb = g.half ? 16 : 4 * elt_bytes(prec);
+    g.tb = prec == MP_FP64 ? 8 : ((prec == MP_FP16 || prec == MP_FP16C) ? 2 : 4);
+    g.tbs = prec == MP_FP32 ? 8 : g.tb;
+    g.kb = prec == MP_FP64 ? 16 : 8;
+    g.Dp = var.DL * var.G;
+    g.HT = pl.H;
+    g.NC = pl.nc;
+    const double side = (double)d * g.sb + (g.half ? d * 16.0 : 0.0) + 2.0 * g.Dp * g.tb;   // st, stp, tw, mup
+    const double key = (double)d * g.kb;
+    const double scr = (double)d * (2.0 * g.tbs + (g.half ? 6.0 : 0.0) + 8.0);             // mu, nrm, flat, T slice
+    const double out = 16.0 * d;                                                            // P, I row window
+    // windows: rows R, columns 3R (Wb = 2R)
+    g.per_R = self ? 4.0 * (side + key) + 3.0 * scr + out : (side + key) + 3.0 * side + 3.0 * scr + out;
+    const int narr = g.half ? 5 : 4;   // st, (stp), tw, mup, keys per side
+    g.fixed = (double)gran * 2.0 /* windows */ * 2.0 /* partial granules */ * narr * (self ? 1 : 2) +
+              2.0 * m * g.Dp * g.tb + 6.0 * scr + (16 << 20);
+    const double avail = (double)budget - g.fixed;
+    int64_t R = avail > 0 ? (int64_t)(avail / g.per_R) : 0;
+    R = R / g.HT * g.HT;
+    if (R < g.HT)
+        return fail(ctx, MP_ERR_NOMEM, "device budget too small for one row segment of the tile plan");
+    R = std::min<int64_t>(R, (n + g.HT - 1) / g.HT * g.HT);
+    g.R = R;
+    g.Wb = std::max<int64_t>(g.NC, (2 * R) / g.NC * g.NC);
+    (void)excl;
+    return MP_OK;
+}
+
+struct Side {
+    VArr st, stp, tw, mup, keys;
+    std::vector<Ivl> valid;   // positions whose precompute is resident
+    Buf scale;
+    const double* T = nullptr;
+};
+
+#define MP_CU(ctx, call)                                                                        \
+    do {                                                                                        \
+        CUresult r_ = (call);                                                                   \
+        if (r_ != CUDA_SUCCESS)                                                                 \
+            return fail((ctx), r_ == CUDA_ERROR_OUT_OF_MEMORY ? MP_ERR_NOMEM : MP_ERR_CUDA,     \
+                        std::string(#call) + ": CUresult " + std::to_string((int)r_));          \
+    } while (0)
+
+struct Streamer {
+    mp_ctx* ctx;
+    cudaStream_t s;
+    Vmm vm;
+    StreamGeo g;
+    int prec;
+    int64_t d, n, m, L;
+    bool self;
+    unsigned char* hkeys = nullptr;        // host key store (pinned), absolute byte layout
+    Buf tslice, mu, nrm, flat, maxbits, dPw, dIw;
+    int64_t wmax = 0;
+    Side sq, sr;
+
+    // granules of array a covering the byte ranges of position intervals (+ trailing positions ex)
+    std::vector<char> need_mask(const VArr& a, const std::vector<Ivl>& iv, double bpp, int64_t ex) const {
+        std::vector<char> nm(a.h.size(), 0);
+        for (const Ivl& x : iv) {
+            const size_t lo = (size_t)(x.first * bpp), hi = std::min(a.bytes, (size_t)((x.second + ex) * bpp));
+            if (hi <= lo) continue;
+            for (size_t gi = lo / vm.gran; gi < (hi + vm.gran - 1) / vm.gran; ++gi) nm[gi] = 1;
+        }
+        return nm;
+    }
+    mp_status remap(VArr& a, const std::vector<char>& nm, bool is_keys, int64_t final_upto) {
+        if (is_keys) {   // save the key granules about to be unmapped (those still accumulating)
+            bool any = false;
+            for (size_t gi = 0; gi < a.h.size(); ++gi) {
+                if (!a.h[gi] || nm[gi]) continue;
+                const size_t b0 = gi * vm.gran;
+                if ((int64_t)((b0 + vm.gran - 1) / (d * g.kb)) < final_upto) { a.saved[gi] = 0; continue; }  // finalized
+                MP_CUDA(ctx, cudaMemcpyAsync(hkeys + b0, (char*)a.ptr() + b0, vm.gran, cudaMemcpyDeviceToHost, s));
+                a.saved[gi] = 1;
+                any = true;
+            }
+            if (any) MP_CUDA(ctx, cudaStreamSynchronize(s));
+        }
+        for (size_t gi = 0; gi < a.h.size(); ++gi)
+            if (a.h[gi] && !nm[gi]) MP_CU(ctx, vm.unmap_g(a, gi));
+        for (size_t gi = 0; gi < a.h.size(); ++gi) {
+            if (a.h[gi] || !nm[gi]) continue;
+            MP_CU(ctx, vm.map_g(a, gi));
+            if (!is_keys) continue;
+            const size_t b0 = gi * vm.gran;
+            if (a.saved[gi]) MP_CUDA(ctx, cudaMemcpyAsync((char*)a.ptr() + b0, hkeys + b0, vm.gran, cudaMemcpyHostToDevice, s));
+            else MP_CUDA(ctx, mpk::launch_init_keys(prec, (char*)a.ptr() + b0, (long long)(vm.gran / g.kb), s));
+        }
+        return MP_OK;
+    }
+    // precompute positions [a, b) of one series (statistics, pair format, seed operands)
+    mp_status precompute(Side& sd, int64_t a, int64_t b) {
+        mpk::PreParams pp{};
+        pp.n = n; pp.d = (int)d; pp.m = (int)m; pp.Dp = g.Dp;
+        const mpk::Variant var = mpk::pick_variant(prec, (int)d);
+        if (var.ctab) { pp.pm_G = var.G; pp.pm_DL = var.DL; }
+        pp.w0 = a; pp.w1 = b;
+        pp.s_off = std::max<int64_t>(0, a - 2);
+        pp.s_end = std::min<int64_t>(n, b + 1);
+        pp.s_ld = pp.s_end - pp.s_off;
+        pp.T_off = pp.s_off;
+        const int64_t len = pp.s_end + m - 1 - pp.s_off;
+        pp.T_ld = len;
+        MP_CUDA(ctx, cudaMemcpy2DAsync(tslice.p, len * 8, sd.T + pp.s_off, L * 8, len * 8, d, cudaMemcpyHostToDevice, s));
+        MP_CUDA(ctx, mpk::launch_check_finite((const double*)tslice.p, d * len, (int*)ctx->flag.p, s));
+        pp.T = (const double*)tslice.p;
+        pp.st = sd.st.ptr(); pp.st_pair = sd.stp.ptr(); pp.tw = sd.tw.ptr(); pp.mup = sd.mup.ptr();
+        pp.mu = mu.p; pp.nrm32 = (float*)nrm.p; pp.nrm64 = (double*)nrm.p; pp.flat = flat.p;
+        pp.scale = (double*)sd.scale.p; pp.maxbits = (unsigned long long*)maxbits.p;
+        MP_CUDA(ctx, mpk::launch_precompute(prec, pp, s, false));
+        return MP_OK;
+    }
+    // per-dimension half-precision scale of one series over all its windows (reading G16)
+    mp_status half_scale(Side& sd) {
+        for (int64_t a = 0; a < n; a += wmax) {
+            const int64_t b = std::min(n, a + wmax);
+            mpk::PreParams pp{};
+            pp.n = n; pp.d = (int)d; pp.m = (int)m;
+            const int64_t len = b + m - 1 - a;
+            pp.w0 = a; pp.w1 = b; pp.T_off = a; pp.T_ld = len;
+            MP_CUDA(ctx, cudaMemcpy2DAsync(tslice.p, len * 8, sd.T + a, L * 8, len * 8, d, cudaMemcpyHostToDevice, s));
+            pp.T = (const double*)tslice.p;
+            pp.maxbits = (unsigned long long*)maxbits.p;
+            pp.scale = (double*)sd.scale.p;
+            MP_CUDA(ctx, mpk::launch_scale_max(pp, a == 0, s));
+            if (b == n) MP_CUDA(ctx, mpk::launch_scale_pick(prec, pp, s));
+        }
+        return MP_OK;
+    }
+    // make the positions `iv` of one series resident (and its keys `kv`: query series only)
+    mp_status ensure_side(Side& sd, std::vector<Ivl> iv, const std::vector<Ivl>* kv, int64_t final_upto) {
+        iv = merge_ivls(iv);
+        const double dd = (double)d;
+        mp_status st;
+        if ((st = remap(sd.st, need_mask(sd.st, iv, dd * g.sb, 0), false, 0)) != MP_OK) return st;
+        if (g.half && (st = remap(sd.stp, need_mask(sd.stp, iv, dd * 16, 1), false, 0)) != MP_OK) return st;
+        if ((st = remap(sd.tw, need_mask(sd.tw, iv, (double)g.Dp * g.tb, m - 1), false, 0)) != MP_OK) return st;
+        if ((st = remap(sd.mup, need_mask(sd.mup, iv, (double)g.Dp * g.tb, 0), false, 0)) != MP_OK) return st;
+        if (kv) {
+            const std::vector<Ivl> kk = merge_ivls(*kv);
+            if ((st = remap(sd.keys, need_mask(sd.keys, kk, dd * g.kb, 0), true, final_upto)) != MP_OK) return st;
+        }
+        const int64_t piece = wmax - 4;   // the window scratch holds R + Wb positions
+        for (const Ivl& x : minus_ivls(iv, sd.valid))
+            for (int64_t a = x.first; a < x.second; a += piece)
+                if ((st = precompute(sd, a, std::min(x.second, a + piece))) != MP_OK) return st;
+        sd.valid = iv;
+        return MP_OK;
+    }
+};
+
+mp_status run_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, int64_t n, int64_t m, int prec,
+                     int64_t excl, int64_t budget, double* P, int64_t* I) {
+    const bool self = Tr == nullptr;
+    if (self && excl < 0) excl = (m + 3) / 4;
+    const int64_t L = n + m - 1;
+    const int64_t H = reseed_interval(ctx, prec, m);
+    const Plan pl = build_plan(d, n, excl, self, prec, H);
+    Streamer S{};
+    S.ctx = ctx;
+    S.s = ctx->stream;
+    S.prec = prec; S.d = d; S.n = n; S.m = m; S.L = L; S.self = self;
+    const std::string err = S.vm.load(ctx->device);
+    if (!err.empty()) return fail(ctx, MP_ERR_UNSUPPORTED, err);
+    mp_status st = plan_stream(ctx, d, n, m, prec, excl, self, budget, S.vm.gran, pl, S.g);
+    if (st != MP_OK) return st;
+    // testing knobs: force a finer geometry (rows rounded to the tile height, diagonals to the
+    // block width) so small inputs exercise many chunks (include/mp.h)
+    if (const char* e = std::getenv("MP_STREAM_ROWS")) {
+        const int64_t r = std::max<int64_t>(1, std::atoll(e));
+        S.g.R = std::max<int64_t>(S.g.HT, (r + S.g.HT - 1) / S.g.HT * S.g.HT);
+    }
+    if (const char* e = std::getenv("MP_STREAM_DIAGS")) {
+        const int64_t w = std::max<int64_t>(1, std::atoll(e));
+        S.g.Wb = std::max<int64_t>(S.g.NC, (w + S.g.NC - 1) / S.g.NC * S.g.NC);
+    }
+    ctx->stream_R = S.g.R;
+    ctx->stream_Wb = S.g.Wb;
+    const StreamGeo& g = S.g;
+    cudaStream_t s = S.s;
+    struct Cleanup {
+        Streamer& S;
+        ~Cleanup() {
+            cudaStreamSynchronize(S.s);
+            S.vm.destroy();
+            if (S.hkeys) cudaFreeHost(S.hkeys);
+            Buf* bs[] = {&S.tslice, &S.mu, &S.nrm, &S.flat, &S.maxbits, &S.dPw, &S.dIw, &S.sq.scale, &S.sr.scale};
+            for (Buf* b : bs) release(*b);
+        }
+    } cleanup{S};
+
+    // window scratch: the largest precompute window is a column window (R + Wb + 1 positions)
+    S.wmax = g.R + g.Wb + 4;
+    const int64_t wmax = S.wmax;
+    MP_CUDA(ctx, ensure(S.tslice, (size_t)d * (wmax + m + 4) * 8));
+    MP_CUDA(ctx, ensure(S.mu, (size_t)d * (wmax + 4) * g.tbs));
+    MP_CUDA(ctx, ensure(S.nrm, (size_t)d * (wmax + 4) * g.tbs));
+    if (g.half) MP_CUDA(ctx, ensure(S.flat, (size_t)d * (wmax + 4) * 3 * 2));
+    MP_CUDA(ctx, ensure(S.maxbits, (size_t)d * 2 * sizeof(unsigned long long)));
+    MP_CUDA(ctx, ensure(S.dPw, (size_t)d * g.R * 8));
+    MP_CUDA(ctx, ensure(S.dIw, (size_t)d * g.R * 8));
+    MP_CUDA(ctx, ensure(ctx->flag, sizeof(int)));
+    MP_CUDA(ctx, cudaMemsetAsync(ctx->flag.p, 0, sizeof(int), s));
+
+    // virtual arrays at full size (absolute-position layout of run_partial)
+    Side* sides[2] = {&S.sq, &S.sr};
+    S.sq.T = T;
+    S.sr.T = Tr;
+    for (int si = 0; si < (self ? 1 : 2); ++si) {
+        Side& sd = *sides[si];
+        MP_CU(ctx, S.vm.reserve_arr(sd.st, (size_t)n * d * g.sb));
+        if (g.half) MP_CU(ctx, S.vm.reserve_arr(sd.stp, (size_t)(n + 1) * d * 16));
+        MP_CU(ctx, S.vm.reserve_arr(sd.tw, (size_t)L * g.Dp * g.tb));
+        MP_CU(ctx, S.vm.reserve_arr(sd.mup, (size_t)n * g.Dp * g.tb));
+        if (g.half) {
+            MP_CUDA(ctx, ensure(sd.scale, (size_t)d * sizeof(double)));
+            if ((st = S.half_scale(sd)) != MP_OK) return st;
+        }
+    }
+    MP_CU(ctx, S.vm.reserve_arr(S.sq.keys, (size_t)n * d * g.kb + 16));
+    MP_CUDA(ctx, cudaHostAlloc((void**)&S.hkeys, S.sq.keys.bytes, cudaHostAllocDefault));
+
+    mpk::MainParams mp{};
+    mp.st_q = S.sq.st.ptr();
+    const Side& rs = self ? S.sq : S.sr;
+    mp.st_r = g.half ? rs.stp.ptr() : rs.st.ptr();
+    mp.tw_q = S.sq.tw.ptr();
+    mp.tw_r = rs.tw.ptr();
+    mp.mu_q = S.sq.mup.ptr();
+    mp.mu_r = rs.mup.ptr();
+    mp.keys = S.sq.keys.ptr();
+    mp.n = n; mp.d = (int)d; mp.m = (int)m; mp.H = (int)H;
+    mp.seed_kahan = prec == MP_FP16CK ? 1 : 0;
+
+    ctx->last_launches = 0;
+    ctx->last_ms = 0.0;
+    std::vector<cudaEvent_t> evs;
+    struct EvFree { std::vector<cudaEvent_t>& v; ~EvFree() { for (auto e : v) cudaEventDestroy(e); } } evfree{evs};
+    const int64_t HT = g.HT, NC = g.NC, nq = std::max<int64_t>(1, (n + HT - 1) / HT), qs = g.R / HT;
+    const int64_t BW = g.Wb / NC;   // blocks per band
+    for (int64_t q0 = 0; q0 < nq; q0 += qs) {
+        const int64_t q1 = std::min(nq, q0 + qs), i0 = q0 * HT, i1 = std::min(n, q1 * HT);
+        for (int64_t B0 = 0; B0 < pl.nb; B0 += BW) {
+            const int64_t B1 = std::min(pl.nb, B0 + BW);
+            const int64_t dlo = pl.dlo + B0 * NC, dhi = std::min(pl.dlo + B1 * NC - 1, pl.dhi);
+            const int64_t ra = std::max(i0, -dhi), rb = std::min(i1, n - dlo);   // rows with cells
+            if (ra >= rb) continue;
+            const Ivl rows{i0, i1}, cols{std::max<int64_t>(0, ra + dlo), std::min<int64_t>(n, rb - 1 + dhi + 1)};
+            MP_CUDA(ctx, cudaStreamSynchronize(s));   // the previous launch is done with the windows
+            if (self) {
+                const std::vector<Ivl> both{rows, cols};
+                if ((st = S.ensure_side(S.sq, both, &both, i0)) != MP_OK) return st;
+            } else {
+                const std::vector<Ivl> r1{rows};
+                if ((st = S.ensure_side(S.sq, r1, &r1, i0)) != MP_OK) return st;
+                if ((st = S.ensure_side(S.sr, {cols}, nullptr, 0)) != MP_OK) return st;
+            }
+            cudaEvent_t e0, e1;
+            MP_CUDA(ctx, cudaEventCreate(&e0));
+            evs.push_back(e0);
+            MP_CUDA(ctx, cudaEventCreate(&e1));
+            evs.push_back(e1);
+            MP_CUDA(ctx, cudaEventRecord(e0, s));
+            if ((st = enqueue_tiles(ctx, s, prec, self, mp, pl, B0, B1, q0, q1, false)) != MP_OK) return st;
+            MP_CUDA(ctx, cudaEventRecord(e1, s));
+        }
+        // rows [i0, i1) are final: later chunks only touch rows >= i1 and (self-join) columns
+        // > their rows.  Their keys are made resident (rows no band reached keep the empty key:
+        // P = +inf, I = -1, reading G3) and finalized.
+        MP_CUDA(ctx, cudaStreamSynchronize(s));
+        if ((st = S.remap(S.sq.keys, S.need_mask(S.sq.keys, {{i0, i1}}, (double)d * g.kb, 0), true, i0)) != MP_OK)
+            return st;
+        const int64_t w = i1 - i0;
+        MP_CUDA(ctx, mpk::launch_finalize_window(prec, S.sq.keys.ptr(), i0, i1, (int)d, (double*)S.dPw.p,
+                                                 (long long*)S.dIw.p, s));
+        MP_CUDA(ctx, cudaMemcpy2DAsync(P + i0, n * 8, S.dPw.p, w * 8, w * 8, d, cudaMemcpyDeviceToHost, s));
+        MP_CUDA(ctx, cudaMemcpy2DAsync(I + i0, n * 8, S.dIw.p, w * 8, w * 8, d, cudaMemcpyDeviceToHost, s));
+    }
+    MP_CUDA(ctx, cudaStreamSynchronize(s));
+    double tot = 0;
+    for (size_t k = 0; k + 1 < evs.size(); k += 2) {
+        float ms = 0.f;
+        MP_CUDA(ctx, cudaEventElapsedTime(&ms, evs[k], evs[k + 1]));
+        tot += ms;
+    }
+    ctx->last_ms = tot;
+    ctx->stream_timed = true;
+    ctx->stream_peak = (int64_t)S.vm.peak;
+    ctx->stream_launches = ctx->last_launches;
+    return finish_partial(ctx, s);
 }
 
 }  // namespace
@@ -328,8 +794,9 @@ mp_status mp_init(mp_ctx** out, const mp_config* cfg) {
         ctx->device = cfg->device;
         for (int i = 0; i < 4; ++i) ctx->H[i] = cfg->reseed_h[i];
         ctx->H[4] = cfg->reseed_h[2];  // FP16C follows FP16
+        ctx->H[5] = cfg->reseed_h[3];  // FP16CK follows MIXED
     }
-    for (int i = 0; i < 5; ++i)
+    for (int i = 0; i < 6; ++i)
         if (ctx->H[i] < 0 || ctx->H[i] > (int64_t(1) << 30)) { delete ctx; return MP_ERR_INVALID; }
     int ndev = 0;
     cudaError_t e = cudaGetDeviceCount(&ndev);
@@ -371,7 +838,7 @@ int64_t mp_key_words(int64_t d, int64_t n, mp_precision prec) {
 
 mp_status mp_plan_bands(int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
                         int self_join, int world, int64_t* block_begin, int64_t* cells) {
-    if (world < 1 || !block_begin || !cells || d < 1 || n < 2 || m < 2 || prec < 0 || prec > 4)
+    if (world < 1 || !block_begin || !cells || d < 1 || n < 2 || m < 2 || prec < 0 || prec > 5)
         return MP_ERR_INVALID;
     if (self_join && exclusion < 0) exclusion = (m + 3) / 4;
     Plan pl = build_plan(d, n, exclusion, self_join != 0, prec, default_h(prec, m));
@@ -388,7 +855,7 @@ mp_status mp_plan_bands(int64_t d, int64_t n, int64_t m, mp_precision prec, int6
 
 mp_status mp_plan_diagonals(int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion,
                             int self_join, int world, int64_t* diag_begin) {
-    if (world < 1 || !diag_begin || d < 1 || n < 2 || m < 2 || prec < 0 || prec > 4) return MP_ERR_INVALID;
+    if (world < 1 || !diag_begin || d < 1 || n < 2 || m < 2 || prec < 0 || prec > 5) return MP_ERR_INVALID;
     if (self_join && exclusion < 0) exclusion = (m + 3) / 4;
     Plan pl = build_plan(d, n, exclusion, self_join != 0, prec, default_h(prec, m));
     if (pl.nb == 0) {
@@ -511,6 +978,7 @@ mp_status mp_selftest_precompute(mp_ctx* ctx, const double* T, int64_t d, int64_
     const mpk::Variant var = mpk::pick_variant(prec, (int)d);
     mpk::PreParams pp{};
     pp.n = n; pp.d = (int)d; pp.m = (int)m; pp.Dp = var.DL * var.G;
+    full_window(pp, n, L);
     if (var.ctab) { pp.pm_G = var.G; pp.pm_DL = var.DL; }
     const size_t eb = elt_bytes(prec), tbs = 8;
     MP_CUDA(ctx, ensure(ctx->nrm, (size_t)n * d * tbs));
@@ -537,12 +1005,53 @@ mp_status mp_last_timing(const mp_ctx* ctx, double* main_kernel_ms, int64_t* lau
     if (!ctx || !main_kernel_ms || !launches) return MP_ERR_INVALID;
     *launches = ctx->last_launches;
     *main_kernel_ms = 0.0;
+    if (ctx->stream_timed) {   // mp_compute_stream: the sum over its launches (measured there)
+        *main_kernel_ms = ctx->last_ms;
+        return MP_OK;
+    }
     if (ctx->last_launches > 0) {
         float ms = 0.f;
         if (cudaEventSynchronize(ctx->ev1) != cudaSuccess) return MP_ERR_CUDA;
         if (cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1) != cudaSuccess) return MP_ERR_CUDA;
         *main_kernel_ms = ms;
     }
+    return MP_OK;
+}
+
+mp_status mp_plan_stream(int64_t d, int64_t n, int64_t m, mp_precision prec, int64_t exclusion, int self_join,
+                         int64_t device_bytes, int64_t granularity, int64_t* rows_per_chunk,
+                         int64_t* diagonals_per_band) {
+    if (!rows_per_chunk || !diagonals_per_band || d < 1 || d > MP_MAX_D || n < 2 || m < 2 || prec < 0 ||
+        prec > 5 || granularity < 1 || device_bytes < 1)
+        return MP_ERR_INVALID;
+    if (self_join && exclusion < 0) exclusion = (m + 3) / 4;
+    const Plan pl = build_plan(d, n, exclusion, self_join != 0, prec, default_h(prec, m));
+    StreamGeo g;
+    mp_status st = plan_stream(nullptr, d, n, m, prec, exclusion, self_join != 0, device_bytes, (size_t)granularity, pl, g);
+    if (st != MP_OK) return st;
+    *rows_per_chunk = g.R;
+    *diagonals_per_band = g.Wb;
+    return MP_OK;
+}
+
+mp_status mp_compute_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, int64_t n, int64_t m,
+                            mp_precision prec, int64_t exclusion, int64_t device_bytes, double* P, int64_t* I) {
+    if (!ctx) return MP_ERR_INVALID;
+    mp_status st = validate(ctx, T, d, n, m, prec);
+    if (st != MP_OK) return st;
+    if (!P || !I) return fail(ctx, MP_ERR_INVALID, "P or I is NULL");
+    if (device_bytes < 1) return fail(ctx, MP_ERR_INVALID, "device_bytes must be positive");
+    MP_CUDA(ctx, cudaSetDevice(ctx->device));
+    return run_stream(ctx, T, Tr, d, n, m, prec, exclusion, device_bytes, P, I);
+}
+
+mp_status mp_last_stream_info(const mp_ctx* ctx, int64_t* rows_per_chunk, int64_t* diagonals_per_band,
+                              int64_t* peak_device_bytes, int64_t* launches) {
+    if (!ctx || !rows_per_chunk || !diagonals_per_band || !peak_device_bytes || !launches) return MP_ERR_INVALID;
+    *rows_per_chunk = ctx->stream_R;
+    *diagonals_per_band = ctx->stream_Wb;
+    *peak_device_bytes = ctx->stream_peak;
+    *launches = ctx->stream_launches;
     return MP_OK;
 }
 

@@ -383,7 +383,7 @@ __device__ __forceinline__ void decode_tile(const MainParams& p, long long t, in
     }
     b = lo;
     const long long delta1 = min(p.delta_lo + b * NC + NC - 1, p.delta_hi);
-    q = max(0ll, -delta1) / p.HT + (t - __ldg(&p.seg_prefix[lo]));
+    q = max(max(0ll, -delta1) / p.HT, p.q_lo) + (t - __ldg(&p.seg_prefix[lo]));
 }
 
 // ------------------------------------------------------------------ tile geometry

@@ -190,7 +190,7 @@ mp_diag_cta_h(const MainParams p) {
 #pragma unroll
         for (int kk = 0; kk < DL; ++kk) QT[kk] = __float2half2_rn((kk * G + g) >= d ? -1.f : 0.f);
         if (lo[0] < hi[0] || lo[1] < hi[1])
-            seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, dP, lo[0] < hi[0], lo[1] < hi[1], lo[0], lo[1], QT);
+            seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, dP, lo[0] < hi[0], lo[1] < hi[1], lo[0], lo[1], QT, p.seed_kahan != 0);
 
         const int nrows = (int)(r1 - r0);
         const int R0 = (int)r0, C0 = (int)(r0 + delta0);  // row / first column of step 0
@@ -212,7 +212,7 @@ mp_diag_cta_h(const MainParams p) {
                 to_seed = H;
                 const long long row = R0 + s0;
                 const bool u0 = row > lo[0] && row < hi[0], u1 = row > lo[1] && row < hi[1];
-                if (u0 || u1) seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, dP, u0, u1, row, row, QT);
+                if (u0 || u1) seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, dP, u0, u1, row, row, QT, p.seed_kahan != 0);
                 seeded_step = s0;
             }
             const int nxt = min(s0 + 2 * SB, nrows);

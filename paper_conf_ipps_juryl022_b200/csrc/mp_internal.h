@@ -32,6 +32,9 @@ struct MainParams {
     int d, m, H;                  // dims, window, re-seed interval H (rows)
     int HT;                       // tile height (multiple of H)
     long long delta_lo, delta_hi; // diagonal range [lo, hi] (j = i + delta)
+    long long q_lo;               // block-major order: first row segment of the launch's row
+                                  // window (0; > 0 only for a streamed chunk, mp_compute_stream)
+    int seed_kahan;               // Mixed kernels: 1 -> Kahan-compensated FP32 seeds (MP_FP16CK)
 };
 
 struct PreParams {
@@ -47,6 +50,12 @@ struct PreParams {
     double* nrm64;
     long long n;
     int d, m;
+    // position window (mp_compute_stream; a full run: w0 = 0, w1 = n, T_off = s_off = 0,
+    // T_ld = L, s_ld = n).  Outputs at absolute positions (st, st_pair, tw, mup) are written for
+    // positions [w0, w1) (tw: t in [w0, w1 + m - 1); st_pair: entries [w0, w1]).  T holds
+    // x[dim][t] at T[dim * T_ld + t - T_off]; the per-window scratch (mu, nrm, flat) holds
+    // position pos at (pos - s_off) with leading dimension s_ld and covers [s_off, s_end).
+    long long w0, w1, T_off, T_ld, s_off, s_end, s_ld;
     // FP16 / Mixed only
     void* st_pair;      // out stats in pair format [pos][dim] (x_pos, x_pos+1) half2 x 4
     double* scale;      // scratch [d]: exact power-of-two per-dimension scale (reading G16)
@@ -55,7 +64,7 @@ struct PreParams {
 };
 
 // Precision codes match mp_precision.
-enum { P64 = 0, P32 = 1, P16 = 2, PMIX = 3, P16C = 4 };
+enum { P64 = 0, P32 = 1, P16 = 2, PMIX = 3, P16C = 4, P16CK = 5 };
 
 // Variant selection for a given (precision, d): dims per lane DL and lanes per cell G.
 struct Variant { int DL; int G; int W; int NC; int cta = 0; /* warps per block of the block-cooperative kernel, 0: warp tiles */
@@ -65,7 +74,15 @@ size_t smem_per_block(int prec, int d, bool self);
 int variant_warps_per_block(int prec, int d, bool self);
 
 // Launchers (return cudaError_t).
-cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s);
+cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s, bool with_scale = true);
+// half modes: per-dimension scale (reading G16) over a window [w0, w1) (reset: clear the maxima
+// first), then pick the scales; mp_compute_stream runs these over every window before the chunks
+cudaError_t launch_scale_max(const PreParams& p, bool reset, cudaStream_t s);
+cudaError_t launch_scale_pick(int prec, const PreParams& p, cudaStream_t s);
+// streamed finalize: keys (internal format, absolute positions) of positions [p0, p1) -> P, I
+// window buffers [rank][p1 - p0]
+cudaError_t launch_finalize_window(int prec, const void* keys, long long p0, long long p1, int d, double* P,
+                                   long long* I, cudaStream_t s);
 cudaError_t launch_init_keys(int prec, void* keys, long long count, cudaStream_t s);
 cudaError_t launch_main(int prec, bool self, const MainParams& p, int grid, cudaStream_t s);
 int main_blocks_per_sm(int prec, int d, bool self);

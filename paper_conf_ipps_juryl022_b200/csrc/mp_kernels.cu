@@ -15,14 +15,14 @@ namespace mpk {
 // L420-444), then df / dg (reading G7) and a = sqrt(2m)/norm (0 for flat windows, G4).
 template <class T>
 __global__ void pre_stats(const PreParams p) {
-    const long long n = p.n;
     const int d = p.d, m = p.m;
-    const long long L = n + m - 1;
+    const long long cntp = p.s_end - p.s_off;   // scratch window [s_off, s_end)
     const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-    if (gid >= n * d) return;
-    const int dim = (int)(gid / n);
-    const long long pos = gid % n;
-    const double* x = p.T + (long long)dim * L + pos;
+    if (gid >= cntp * d) return;
+    const int dim = (int)(gid / cntp);
+    const long long pos = p.s_off + gid % cntp;
+    const long long so = (long long)dim * p.s_ld + (pos - p.s_off);
+    const double* x = p.T + (long long)dim * p.T_ld + (pos - p.T_off);
     // two-pass with compensated (Kahan) sums in the precalc precision; the paper leaves the
     // precalculation formulas out and stresses its accuracy (L792-794)
     T s = 0, c = 0;
@@ -42,25 +42,24 @@ __global__ void pre_stats(const PreParams p) {
         c = (tt - q) - y;
         q = tt;
     }
-    reinterpret_cast<T*>(p.mu)[(long long)dim * n + pos] = mu;
+    reinterpret_cast<T*>(p.mu)[so] = mu;
     const T nr = sqrt(q);
-    if constexpr (sizeof(T) == 4) p.nrm32[(long long)dim * n + pos] = nr; else p.nrm64[(long long)dim * n + pos] = nr;
+    if constexpr (sizeof(T) == 4) p.nrm32[so] = nr; else p.nrm64[so] = nr;
 }
 
 template <class T, class A = T>  // A: precalc arithmetic (FP32 mode: FP64, reading R1)
 __global__ void pre_diff(const PreParams p) {
     using V4 = typename PT<T>::V4;
-    const long long n = p.n;
     const int d = p.d, m = p.m;
-    const long long L = n + m - 1;
     const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-    if (gid >= n * d) return;
-    const long long pos = gid / d;  // position-major output
+    if (gid >= (p.w1 - p.w0) * d) return;
+    const long long pos = p.w0 + gid / d;  // position-major output
     const int dim = (int)(gid % d);
-    const double* x = p.T + (long long)dim * L;
-    const A* mu = reinterpret_cast<const A*>(p.mu) + (long long)dim * n;
+    const double* x = p.T + (long long)dim * p.T_ld - p.T_off;                    // x[t]
+    const A* mu = reinterpret_cast<const A*>(p.mu) + (long long)dim * p.s_ld - p.s_off;  // mu[pos]
+    const long long so = (long long)dim * p.s_ld + (pos - p.s_off);
     A nr;
-    if constexpr (sizeof(A) == 4) nr = p.nrm32[(long long)dim * n + pos]; else nr = p.nrm64[(long long)dim * n + pos];
+    if constexpr (sizeof(A) == 4) nr = p.nrm32[so]; else nr = p.nrm64[so];
     V4 v;
     if (pos == 0) {
         v.x = 0; v.y = 0;
@@ -78,18 +77,17 @@ __global__ void pre_diff(const PreParams p) {
 // (the seeds' operands: a lane's dims are contiguous, so they load as vectors)
 template <class T, class A = T>
 __global__ void pre_pm(const PreParams p) {
-    const long long n = p.n, L = p.n + p.m - 1;
     const int d = p.d, Dp = p.Dp;
     const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-    if (gid >= L * Dp) return;
-    const long long t = gid / Dp;
+    if (gid >= (p.w1 + p.m - 1 - p.w0) * Dp) return;
+    const long long t = p.w0 + gid / Dp;
     const int dim = (int)(gid % Dp);
     T* tw = reinterpret_cast<T*>(p.tw);
     T* mup = reinterpret_cast<T*>(p.mup);
     // pm_G > 0: dim kk*G + g is stored at g*DL + kk (each lane's dims contiguous)
     const long long o = p.pm_G > 0 ? t * Dp + (dim % p.pm_G) * p.pm_DL + dim / p.pm_G : gid;
-    tw[o] = dim < d ? (T)p.T[(long long)dim * L + t] : (T)0;
-    if (t < n) mup[o] = dim < d ? (T)reinterpret_cast<const A*>(p.mu)[(long long)dim * n + t] : (T)0;
+    tw[o] = dim < d ? (T)p.T[(long long)dim * p.T_ld + (t - p.T_off)] : (T)0;
+    if (t < p.w1) mup[o] = dim < d ? (T)reinterpret_cast<const A*>(p.mu)[(long long)dim * p.s_ld + (t - p.s_off)] : (T)0;
 }
 
 // ------------------------------------------------------------------ precompute, FP16 / Mixed
@@ -97,13 +95,13 @@ __global__ void pre_pm(const PreParams p) {
 // window energies (QT, norm^2) <= 2^14 (and, for FP16, the window sums <= 2^14); z-normalised
 // distances are invariant under it (pinned in tests/test_oracle.py).
 __global__ void pre_scale_max(const PreParams p) {
-    const long long n = p.n, L = p.n + p.m - 1;
     const int d = p.d, m = p.m;
+    const long long cntp = p.w1 - p.w0;
     const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-    if (gid >= n * d) return;
-    const int dim = (int)(gid / n);
-    const long long pos = gid % n;
-    const double* x = p.T + (long long)dim * L + pos;
+    if (gid >= cntp * d) return;
+    const int dim = (int)(gid / cntp);
+    const long long pos = p.w0 + gid % cntp;
+    const double* x = p.T + (long long)dim * p.T_ld + (pos - p.T_off);
     double s = 0, amax = 0;
     for (int t = 0; t < m; ++t) { s += x[t]; amax = fmax(amax, fabs(x[t])); }
     const double mu = s / m;
@@ -123,18 +121,20 @@ __global__ void pre_scale_pick(const PreParams p, int pure16) {
     e = max(-60, min(60, e));
     p.scale[dim] = ldexp(1.0, e);
 }
-template <class T, bool KAHAN = false>  // T = float (Mixed) or __half (FP16; FP16C: KAHAN)
+// T = float: Mixed (plain FP32 sums, L777-785) or FP16CK (KAHAN: FP32 with Kahan-compensated
+// sums, the text's FP16C reading L786-791); T = __half: FP16 or FP16C (KAHAN, Fig. 1 reading)
+template <class T, bool KAHAN = false>
 __global__ void pre_stats_h(const PreParams p) {
-    const long long n = p.n, L = p.n + p.m - 1;
     const int d = p.d, m = p.m;
+    const long long cntp = p.s_end - p.s_off;   // scratch window [s_off, s_end)
     const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-    if (gid >= n * d) return;
-    const int dim = (int)(gid / n);
-    const long long pos = gid % n;
+    if (gid >= cntp * d) return;
+    const int dim = (int)(gid / cntp);
+    const long long pos = p.s_off + gid % cntp;
     const double sc = p.scale[dim];
-    const double* x = p.T + (long long)dim * L + pos;
+    const double* x = p.T + (long long)dim * p.T_ld + (pos - p.T_off);
     T mu, nr;
-    if constexpr (sizeof(T) == 4) {  // compensated, as in FP32 mode
+    if constexpr (sizeof(T) == 4 && KAHAN) {  // FP16CK: FP32 two-pass, Kahan-compensated sums
         float s = 0, c = 0;
         for (int t = 0; t < m; ++t) { const float y = (float)(sc * x[t]) - c; const float tt = s + y; c = (tt - s) - y; s = tt; }
         mu = s / (float)m;
@@ -143,6 +143,16 @@ __global__ void pre_stats_h(const PreParams p) {
         for (int t = 0; t < m; ++t) {
             const float cx = (float)(sc * x[t]) - mu;
             const float y = cx * cx - c; const float tt = q + y; c = (tt - q) - y; q = tt;
+        }
+        nr = sqrtf(q);
+    } else if constexpr (sizeof(T) == 4) {  // Mixed: FP32 two-pass, plain sums
+        float s = 0;
+        for (int t = 0; t < m; ++t) s += (float)(sc * x[t]);
+        mu = s / (float)m;
+        float q = 0;
+        for (int t = 0; t < m; ++t) {
+            const float cx = (float)(sc * x[t]) - mu;
+            q = fmaf(cx, cx, q);
         }
         nr = sqrtf(q);
     } else if constexpr (!KAHAN) {  // FP16 mode: plain half arithmetic (the paper's FP16 precalc)
@@ -175,21 +185,21 @@ __global__ void pre_stats_h(const PreParams p) {
         }
         nr = hsqrt(q);
     }
-    reinterpret_cast<T*>(p.mu)[(long long)dim * n + pos] = mu;
-    reinterpret_cast<T*>(p.nrm32)[(long long)dim * n + pos] = nr;   // typed scratch
+    reinterpret_cast<T*>(p.mu)[(long long)dim * p.s_ld + (pos - p.s_off)] = mu;
+    reinterpret_cast<T*>(p.nrm32)[(long long)dim * p.s_ld + (pos - p.s_off)] = nr;   // typed scratch
 }
 template <class T>
 __global__ void pre_diff_h(const PreParams p) {
-    const long long n = p.n, L = p.n + p.m - 1;
     const int d = p.d, m = p.m;
+    const long long f0 = p.w0 > 0 ? p.w0 - 1 : 0;   // flat scratch for [f0, s_end) (pre_fmt_h)
     const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-    if (gid >= n * d) return;
-    const long long pos = gid / d;
+    if (gid >= (p.s_end - f0) * d) return;
+    const long long pos = f0 + gid / d;
     const int dim = (int)(gid % d);
     const double sc = p.scale[dim];
-    const double* x = p.T + (long long)dim * L;
-    const T* mu = reinterpret_cast<const T*>(p.mu) + (long long)dim * n;
-    const T nr = reinterpret_cast<const T*>(p.nrm32)[(long long)dim * n + pos];
+    const double* x = p.T + (long long)dim * p.T_ld - p.T_off;                       // x[t]
+    const T* mu = reinterpret_cast<const T*>(p.mu) + (long long)dim * p.s_ld - p.s_off;  // mu[pos]
+    const T nr = reinterpret_cast<const T*>(p.nrm32)[(long long)dim * p.s_ld + (pos - p.s_off)];
     __half* flat = reinterpret_cast<__half*>(p.flat);
     float df = 0, dg = 0, av;
     if constexpr (sizeof(T) == 4) {
@@ -208,10 +218,10 @@ __global__ void pre_diff_h(const PreParams p) {
         av = __half2float(nr) > 0.f ? __half2float(__hdiv(hsqrt(__int2half_rn(2 * m)), nr)) : 0.f;
     }
     av = fminf(av, 65504.f);  // finite half (near-flat windows)
-    const long long o = pos * d + dim;
+    const long long o = (pos - p.s_off) * d + dim, nd = p.s_ld * d;
     flat[o] = __float2half_rn(df);
-    flat[n * d + o] = __float2half_rn(dg);
-    flat[2 * n * d + o] = __float2half_rn(av);
+    flat[nd + o] = __float2half_rn(dg);
+    flat[2 * nd + o] = __float2half_rn(av);
 }
 // row format (x, x) and pair format (x_pos, x_pos+1) H4 entries for the half2 kernel.  The
 // pair array has n+1 entries: entry e holds (x_{e-1}, x_e), so a pair starting at column -1
@@ -220,43 +230,43 @@ __global__ void pre_fmt_h(const PreParams p) {
     const long long n = p.n;
     const int d = p.d;
     const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-    if (gid >= (n + 1) * d) return;
-    const long long e = gid / d;          // pair entry; first position e - 1
+    if (gid >= (p.w1 - p.w0 + 1) * d) return;   // pair entries [w0, w1]
+    const long long e = p.w0 + gid / d;          // pair entry; first position e - 1
     const int dim = (int)(gid % d);
     const __half* f = reinterpret_cast<const __half*>(p.flat);
-    const long long nd = n * d;
+    const long long nd = p.s_ld * d;
     const __half z = __float2half(0.f);
-    const long long ia = (e - 1) * d + dim, ib = e * d + dim;
+    const long long ia = (e - 1 - p.s_off) * d + dim, ib = (e - p.s_off) * d + dim;
     const bool va = e >= 1, vb = e < n;
     H4 q;
     q.x = __halves2half2(va ? f[ia] : z, vb ? f[ib] : z);
     q.y = __halves2half2(va ? f[nd + ia] : z, vb ? f[nd + ib] : z);
     q.z = __halves2half2(va ? f[2 * nd + ia] : z, vb ? f[2 * nd + ib] : z);
     q.w = __half2half2(z);
-    reinterpret_cast<H4*>(p.st_pair)[gid] = q;
-    if (vb) {  // row format: one position (the kernel broadcasts it to both cells of a pair)
+    reinterpret_cast<H4*>(p.st_pair)[e * d + dim] = q;
+    if (vb && e < p.w1) {  // row format: one position (the kernel broadcasts it to both cells of a pair)
         RH r;
         r.df = f[ib]; r.dg = f[nd + ib]; r.a = f[2 * nd + ib]; r.t = z;
-        reinterpret_cast<RH*>(p.st)[ib] = r;
+        reinterpret_cast<RH*>(p.st)[e * d + dim] = r;
     }
 }
 template <class T>
 __global__ void pre_pm_h(const PreParams p) {
-    const long long n = p.n, L = p.n + p.m - 1;
     const int d = p.d, Dp = p.Dp;
-    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-    if (gid >= L * Dp) return;
+    const long long gid0 = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    if (gid0 >= (p.w1 + p.m - 1 - p.w0) * Dp) return;
+    const long long gid = p.w0 * Dp + gid0;       // absolute [t][Dp] index
     const long long t = gid / Dp;
     const int dim = (int)(gid % Dp);
     T* tw = reinterpret_cast<T*>(p.tw);
     T* mup = reinterpret_cast<T*>(p.mup);
     if (dim < d) {
-        const double v = p.scale[dim] * p.T[(long long)dim * L + t];
+        const double v = p.scale[dim] * p.T[(long long)dim * p.T_ld + (t - p.T_off)];
         if constexpr (sizeof(T) == 4) tw[gid] = (float)v; else tw[gid] = __double2half(v);
     } else {
         tw[gid] = (T)0.f;
     }
-    if (t < n) mup[gid] = dim < d ? reinterpret_cast<const T*>(p.mu)[(long long)dim * n + t] : (T)0.f;
+    if (t < p.w1) mup[gid] = dim < d ? reinterpret_cast<const T*>(p.mu)[(long long)dim * p.s_ld + (t - p.s_off)] : (T)0.f;
 }
 
 // ------------------------------------------------------------------ keys
@@ -309,6 +319,36 @@ __global__ void finalize64(const long long* ext, long long n, int d, double* P, 
     P[(long long)rk * n + pos] = pv;
     I[(long long)rk * n + pos] = oi;
 }
+// streamed finalize (mp_compute_stream): internal keys of positions [p0, p1) -> window buffers
+// P, I [rank][p1 - p0]; same arithmetic as finalize32 / keys64_to_ext + finalize64
+__global__ void finalize_window32(const unsigned long long* k, long long p0, long long p1, int d, double* P, long long* I) {
+    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    const long long w = p1 - p0;
+    if (gid >= w * d) return;
+    const long long pos = p0 + gid / d;
+    const int rk = (int)(gid % d);
+    const unsigned long long key = k[pos * d + rk];
+    double pv;
+    long long ix;
+    if (key >= EMPTY32) { pv = __longlong_as_double(0x7ff0000000000000ll); ix = -1; }
+    else { pv = (double)__uint_as_float((unsigned)(key >> 32)) / (double)(rk + 1); ix = (long long)(unsigned)key; }
+    P[(long long)rk * w + (pos - p0)] = pv;
+    I[(long long)rk * w + (pos - p0)] = ix;
+}
+__global__ void finalize_window64(const K64* k, long long p0, long long p1, int d, double* P, long long* I) {
+    const long long gid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    const long long w = p1 - p0;
+    if (gid >= w * d) return;
+    const long long pos = p0 + gid / d;
+    const int rk = (int)(gid % d);
+    const K64 key = k[pos * d + rk];
+    double pv;
+    long long oi;
+    if (key.v >= EMPTY64V) { pv = __longlong_as_double(0x7ff0000000000000ll); oi = -1; }
+    else { pv = __longlong_as_double((long long)key.v) / (double)(rk + 1); oi = (long long)key.i; }
+    P[(long long)rk * w + (pos - p0)] = pv;
+    I[(long long)rk * w + (pos - p0)] = oi;
+}
 __global__ void check_finite(const double* x, long long count, int* flag) {
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < count;
          i += (long long)gridDim.x * blockDim.x)
@@ -321,6 +361,7 @@ static inline unsigned grid1d(long long count, int bs) { return (unsigned)((coun
 Variant pick_variant(int prec, int d) {
     // A lane holds DL <= 16 dims (register budget; DL = 32 only for FP32 d > 512); for small
     // d a lane owns W = 2 adjacent diagonals (d <= 8).
+    if (prec == P16CK) prec = PMIX;   // same kernels as Mixed
     int dp = 1;
     while (dp < d) dp <<= 1;
     Variant v;
@@ -470,6 +511,7 @@ static long long dispatch_cta64(int op, int G, const MainParams* p, int grid, cu
 }
 
 static long long dispatch(int op, int prec, bool self, int d, const MainParams* p, int grid, cudaStream_t s) {
+    if (prec == P16CK) prec = PMIX;   // the Mixed kernels; the seed compensation is MainParams::seed_kahan
     const Variant v = pick_variant(prec, d);
     if (v.cta && (prec == P16 || prec == PMIX || prec == P16C)) {
         const int md = prec == P16 ? 0 : prec == PMIX ? 1 : 2;
@@ -495,39 +537,56 @@ cudaError_t launch_main(int prec, bool self, const MainParams& p, int grid, cuda
     return (cudaError_t)dispatch(1, prec, self, p.d, &p, grid, s);
 }
 
-cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s) {
-    const long long cnt = p.n * p.d;
-    const long long L = p.n + p.m - 1;
+cudaError_t launch_scale_max(const PreParams& p, bool reset, cudaStream_t s) {
+    if (reset) cudaMemsetAsync(p.maxbits, 0, 2 * p.d * sizeof(unsigned long long), s);
+    pre_scale_max<<<grid1d((p.w1 - p.w0) * p.d, 256), 256, 0, s>>>(p);
+    return cudaGetLastError();
+}
+cudaError_t launch_scale_pick(int prec, const PreParams& p, cudaStream_t s) {
+    pre_scale_pick<<<grid1d(p.d, 128), 128, 0, s>>>(p, (prec == PMIX || prec == P16CK) ? 0 : 1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s, bool with_scale) {
+    const long long cs = (p.s_end - p.s_off) * p.d;          // window statistics (scratch)
+    const long long cw = (p.w1 - p.w0) * p.d;                // stats entries written
+    const long long cpm = (p.w1 + p.m - 1 - p.w0) * p.Dp;    // seed operands written
     if (prec == P64) {
-        pre_stats<double><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-        pre_diff<double><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-        pre_pm<double><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
+        pre_stats<double><<<grid1d(cs, 256), 256, 0, s>>>(p);
+        pre_diff<double><<<grid1d(cw, 256), 256, 0, s>>>(p);
+        pre_pm<double><<<grid1d(cpm, 256), 256, 0, s>>>(p);
     } else if (prec == P32) {
         // FP32 mode: window stats and df / dg / a in FP64 from the FP64 input, rounded once to
         // FP32 (reading R1'): FP32 cancellation in x - mu grows with the window's offset.
         // (FP64 seeds from the FP64 series were measured too: no accuracy gain, C2 +11 %.)
-        pre_stats<double><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-        pre_diff<float, double><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-        pre_pm<float, double><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
+        pre_stats<double><<<grid1d(cs, 256), 256, 0, s>>>(p);
+        pre_diff<float, double><<<grid1d(cw, 256), 256, 0, s>>>(p);
+        pre_pm<float, double><<<grid1d(cpm, 256), 256, 0, s>>>(p);
     } else {
-        const bool mixed = prec == PMIX;
-        cudaMemsetAsync(p.maxbits, 0, 2 * p.d * sizeof(unsigned long long), s);
-        pre_scale_max<<<grid1d(cnt, 256), 256, 0, s>>>(p);
-        pre_scale_pick<<<grid1d(p.d, 128), 128, 0, s>>>(p, mixed ? 0 : 1);
-        if (mixed) {
-            pre_stats_h<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-            pre_diff_h<float><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-            pre_pm_h<float><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
-        } else if (prec == P16C) {
-            pre_stats_h<__half, true><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-            pre_diff_h<__half><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-            pre_pm_h<__half><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
-        } else {
-            pre_stats_h<__half><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-            pre_diff_h<__half><<<grid1d(cnt, 256), 256, 0, s>>>(p);
-            pre_pm_h<__half><<<grid1d(L * p.Dp, 256), 256, 0, s>>>(p);
+        if (with_scale) {  // a streamed run computes the per-dimension scale over all windows first
+            launch_scale_max(p, true, s);
+            launch_scale_pick(prec, p, s);
         }
-        pre_fmt_h<<<grid1d((p.n + 1) * p.d, 256), 256, 0, s>>>(p);
+        const long long f0 = p.w0 > 0 ? p.w0 - 1 : 0;
+        const long long cf = (p.s_end - f0) * p.d;          // flat scratch (pre_diff_h)
+        if (prec == P16CK) {
+            pre_stats_h<float, true><<<grid1d(cs, 256), 256, 0, s>>>(p);
+            pre_diff_h<float><<<grid1d(cf, 256), 256, 0, s>>>(p);
+            pre_pm_h<float><<<grid1d(cpm, 256), 256, 0, s>>>(p);
+        } else if (prec == PMIX) {
+            pre_stats_h<float><<<grid1d(cs, 256), 256, 0, s>>>(p);
+            pre_diff_h<float><<<grid1d(cf, 256), 256, 0, s>>>(p);
+            pre_pm_h<float><<<grid1d(cpm, 256), 256, 0, s>>>(p);
+        } else if (prec == P16C) {
+            pre_stats_h<__half, true><<<grid1d(cs, 256), 256, 0, s>>>(p);
+            pre_diff_h<__half><<<grid1d(cf, 256), 256, 0, s>>>(p);
+            pre_pm_h<__half><<<grid1d(cpm, 256), 256, 0, s>>>(p);
+        } else {
+            pre_stats_h<__half><<<grid1d(cs, 256), 256, 0, s>>>(p);
+            pre_diff_h<__half><<<grid1d(cf, 256), 256, 0, s>>>(p);
+            pre_pm_h<__half><<<grid1d(cpm, 256), 256, 0, s>>>(p);
+        }
+        pre_fmt_h<<<grid1d((p.w1 - p.w0 + 1) * p.d, 256), 256, 0, s>>>(p);
     }
     return cudaGetLastError();
 }
@@ -544,6 +603,14 @@ cudaError_t launch_keys_to_ext(int prec, const void* keys, void* ext, long long 
         return cudaGetLastError();
     }
     return cudaMemcpyAsync(ext, keys, count * sizeof(long long), cudaMemcpyDeviceToDevice, s);
+}
+
+cudaError_t launch_finalize_window(int prec, const void* keys, long long p0, long long p1, int d, double* P,
+                                   long long* I, cudaStream_t s) {
+    const long long cnt = (p1 - p0) * d;
+    if (prec == P64) finalize_window64<<<grid1d(cnt, 256), 256, 0, s>>>(reinterpret_cast<const K64*>(keys), p0, p1, d, P, I);
+    else finalize_window32<<<grid1d(cnt, 256), 256, 0, s>>>(reinterpret_cast<const unsigned long long*>(keys), p0, p1, d, P, I);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_key_mask(long long count, long long* ext, const long long* gv, cudaStream_t s) {

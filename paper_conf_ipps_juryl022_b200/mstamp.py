@@ -18,13 +18,13 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("MP_LIB_PATH") or os.path.join(_HERE, "lib", "libmstamp_b200.so")
 
-PRECISIONS = {"fp64": 0, "fp32": 1, "fp16": 2, "mixed": 3, "fp16c": 4}
+PRECISIONS = {"fp64": 0, "fp32": 1, "fp16": 2, "mixed": 3, "fp16c": 4, "fp16ck": 5}
 STATUS = {0: "MP_OK", 1: "MP_ERR_INVALID", 2: "MP_ERR_NOMEM", 3: "MP_ERR_CUDA", 4: "MP_ERR_NCCL",
           5: "MP_ERR_UNSUPPORTED"}
 EXPORTS = ["mp_init", "mp_free", "mp_last_error", "mp_version", "mp_compute", "mp_compute_device",
            "mp_key_words", "mp_partial_device", "mp_key_mask_device", "mp_finalize_device",
            "mp_plan_bands", "mp_plan_diagonals", "mp_last_timing", "mp_selftest_sort_scan",
-           "mp_selftest_precompute"]
+           "mp_selftest_precompute", "mp_compute_stream", "mp_plan_stream", "mp_last_stream_info"]
 
 _lib = None
 
@@ -78,6 +78,12 @@ def load():
     lib.mp_selftest_sort_scan.restype = i32
     lib.mp_selftest_precompute.argtypes = [p, p, i64, i64, i64, i32, p, p, p]
     lib.mp_selftest_precompute.restype = i32
+    lib.mp_compute_stream.argtypes = [p, p, p, i64, i64, i64, i32, i64, i64, p, p]
+    lib.mp_compute_stream.restype = i32
+    lib.mp_plan_stream.argtypes = [i64, i64, i64, i32, i64, i32, i64, i64, p, p]
+    lib.mp_plan_stream.restype = i32
+    lib.mp_last_stream_info.argtypes = [p, p, p, p, p]
+    lib.mp_last_stream_info.restype = i32
     _lib = lib
     return lib
 
@@ -113,6 +119,19 @@ def plan_diagonals(d, n, m, prec="fp32", exclusion=-1, self_join=True, world=1):
     if st != 0:
         raise MPError(st, "mp_plan_diagonals")
     return db
+
+
+def plan_stream(d, n, m, prec="fp32", exclusion=-1, self_join=True, device_bytes=1 << 30,
+                granularity=2 << 20):
+    """Host scheduler of mp_compute_stream: (rows per chunk R, diagonals per band Wb)."""
+    lib = load()
+    out = np.zeros(2, dtype=np.int64)
+    st = lib.mp_plan_stream(d, n, m, _prec(prec), exclusion, int(bool(self_join)), int(device_bytes),
+                            int(granularity), out[0:].ctypes.data_as(ctypes.c_void_p),
+                            out[1:].ctypes.data_as(ctypes.c_void_p))
+    if st != 0:
+        raise MPError(st, "mp_plan_stream")
+    return int(out[0]), int(out[1])
 
 
 def key_words(d, n, prec="fp32") -> int:
@@ -206,6 +225,44 @@ class Context:
                                P.ctypes.data_as(ctypes.c_void_p), I.ctypes.data_as(ctypes.c_void_p))
         self._check(st, "mp_compute")
         return P, I
+
+    def compute_stream(self, T, m, prec="fp32", exclusion=-1, Tr=None, device_bytes=1 << 30, out=None):
+        """Beyond-memory streaming (mp_compute_stream): the same P, I as compute() with at most
+        about device_bytes of device memory for the per-position arrays."""
+        T = np.ascontiguousarray(T, dtype=np.float64)
+        if T.ndim == 1:
+            T = T[None, :]
+        d, L = T.shape
+        n = L - m + 1
+        Tr_ = None
+        if Tr is not None:
+            Tr_ = np.ascontiguousarray(Tr, dtype=np.float64)
+            if Tr_.ndim == 1:
+                Tr_ = Tr_[None, :]
+            if Tr_.shape != T.shape:
+                raise MPError(1, "AB-join needs equal shapes")
+        if out is None:
+            P = np.empty((d, n), dtype=np.float64)
+            I = np.empty((d, n), dtype=np.int64)
+        else:
+            P, I = out
+            if (P.shape != (d, n) or I.shape != (d, n) or P.dtype != np.float64 or I.dtype != np.int64
+                    or not P.flags.c_contiguous or not I.flags.c_contiguous):
+                raise MPError(1, "out must be C-contiguous float64 / int64 arrays of shape (d, n)")
+        st = load().mp_compute_stream(self._ctx, T.ctypes.data_as(ctypes.c_void_p),
+                                      None if Tr_ is None else Tr_.ctypes.data_as(ctypes.c_void_p),
+                                      d, n, m, _prec(prec), int(exclusion), int(device_bytes),
+                                      P.ctypes.data_as(ctypes.c_void_p), I.ctypes.data_as(ctypes.c_void_p))
+        self._check(st, "mp_compute_stream")
+        return P, I
+
+    def last_stream_info(self):
+        """(rows per chunk, diagonals per band, peak mapped device bytes, launches) of the last
+        compute_stream."""
+        v = np.zeros(4, dtype=np.int64)
+        ptr = [ctypes.c_void_p(v.ctypes.data + 8 * k) for k in range(4)]
+        self._check(load().mp_last_stream_info(self._ctx, *ptr), "mp_last_stream_info")
+        return tuple(int(x) for x in v)
 
     # ---- device memory (torch tensors)
     def compute_device(self, T, m, P, I, prec="fp32", exclusion=-1, Tr=None, stream=None):

@@ -20,7 +20,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 from paper_conf_ipps_juryl022_b200 import datagen, mstamp  # noqa: E402
 
-MODES = ["fp64", "fp32", "mixed", "fp16c", "fp16"]
+MODES = ["fp64", "fp32", "mixed", "fp16ck", "fp16c", "fp16"]
 RELAX = [0.0, 0.01, 0.05, 0.1]
 
 

@@ -21,7 +21,7 @@ import torch  # noqa: E402
 import oracle  # noqa: E402  (test infrastructure: the checker, never the product path)
 from paper_conf_ipps_juryl022_b200 import datagen, mstamp  # noqa: E402
 
-MODES = ["mixed", "fp16c", "fp16"]
+MODES = ["mixed", "fp16ck", "fp16c", "fp16"]
 
 
 def stats(err, scale):
