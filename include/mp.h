@@ -69,7 +69,17 @@ typedef struct {
                                (also FP16CK);
                                0 -> default (R2); rounded up to a multiple of 8 (re-seeds
                                fall on staging-batch starts); < 0 or > 2^30 -> MP_ERR_INVALID */
+    int seed_mode;          /* how the QT seeds of MIXED / FP16CK are computed:
+                               MP_SEEDS_DIRECT (0): per-cell dot products on the CUDA cores, in
+                               FP32; MP_SEEDS_TC (1): one tensor-core GEMM per row chunk
+                               (tcgen05, FP16 operands, FP32 accumulation; SURVEY 8(f) NEXT-3,
+                               PAPER.md:L2433-2434) for the block kernels (d >= 64), written to a
+                               seed table the fused kernel reads.  Other precisions ignore it.
+                               Other values -> MP_ERR_INVALID. */
 } mp_config;
+
+#define MP_SEEDS_DIRECT 0
+#define MP_SEEDS_TC 1
 
 /* Create a context on cfg->device (cfg == NULL -> device 0, defaults). */
 mp_status mp_init(mp_ctx** out, const mp_config* cfg);
@@ -197,6 +207,15 @@ mp_status mp_last_stream_info(const mp_ctx* ctx, int64_t* rows_per_chunk, int64_
  *   returned -- FP64 and FP32 only).
  */
 mp_status mp_selftest_sort_scan(mp_ctx* ctx, int64_t d, int64_t count, const float* in, float* out);
+/* mp_selftest_seeds: the tensor-core seed GEMM (MP_SEEDS_TC) alone: after the MIXED / FP16CK
+ *   precalculation (prec) of T (and Tr; NULL: self-join), the seeds QT(r H, j) of the rows
+ *   r in [r_lo, r_hi) against every column j in [0, n), for every dimension, in the precalc's
+ *   scaled units (x s_k, reading G16).  out: (r_hi - r_lo) x d x n doubles, [r][dim][j] (the half
+ *   values the fused kernel would read).  scale_out: d doubles, the per-dimension scale of T
+ *   (of Tr: multiply by Tr's scale, returned in scale_out[d .. 2d) for an AB-join). */
+mp_status mp_selftest_seeds(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, int64_t n, int64_t m,
+                            mp_precision prec, int64_t H, int64_t r_lo, int64_t r_hi, double* out,
+                            double* scale_out);
 mp_status mp_selftest_precompute(mp_ctx* ctx, const double* T, int64_t d, int64_t n, int64_t m,
                                  mp_precision prec, double* df, double* dg, double* a);
 

@@ -23,7 +23,7 @@ NVCC = os.environ.get("NVCC", "nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC", "-I", os.path.join(HERE, "..", "include")]
 
-SOURCES = ["mp_kernels.cu", "mp_api.cpp"]
+SOURCES = ["mp_kernels.cu", "mp_seed_tc.cu", "mp_api.cpp"]
 
 
 def _sources():

@@ -10,6 +10,7 @@
 #include "mp_internal.h"
 
 #include <cuda.h>           // driver-API types only (VMM entry points are fetched at run time)
+#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -48,7 +49,9 @@ struct mp_ctx {
     std::string err;
     // cached scratch
     Buf dT, dTr, st_q, st_r, tw_q, tw_r, mu_q, mu_r, mup_q, mup_r, nrm, keys, ext, seg, counter, dP, dI, flag;
-    Buf stp_q, stp_r, scale, maxbits, flat;  // FP16 / Mixed precompute
+    Buf stp_q, stp_r, scale, scale_r, maxbits, flat;  // FP16 / Mixed precompute
+    Buf seedtab;            // tensor-core seed table (seed_mode MP_SEEDS_TC)
+    int seed_mode = MP_SEEDS_DIRECT;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     int* hflag = nullptr;   // pinned read-back of the non-finite flag
     double last_ms = 0.0;
@@ -248,6 +251,12 @@ mp_status enqueue_tiles(mp_ctx* ctx, cudaStream_t s, int prec, bool self, mpk::M
     return MP_OK;
 }
 
+// Tensor-core seeds apply to the FP32-precalc half modes (Mixed, FP16CK) on the block kernels.
+constexpr int64_t kSeedTabBytes = int64_t(1) << 30;   // seed table per row chunk (device bytes)
+bool tc_seeds(const mp_ctx* ctx, int prec) {
+    return ctx->seed_mode == MP_SEEDS_TC && (prec == MP_MIXED || prec == MP_FP16CK);
+}
+
 // Re-seed interval of a run: the context's (mp_config.reseed_h) or the default, rounded up to a
 // multiple of 8 (every kernel steps in batches of 1, 2 or 4 rows, so every re-seed row
 // i = 0 mod H is a batch start in every kernel variant; include/mp.h, mp_config.reseed_h).
@@ -258,7 +267,7 @@ int64_t reseed_interval(const mp_ctx* ctx, int prec, int64_t m) {
 
 // Device pipeline: keys for band (rank, world) of the tile plan, internal key format.
 mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const double* dTr, int64_t d,
-                      int64_t n, int64_t m, int prec, int64_t excl, int rank, int world) {
+                      int64_t n, int64_t m, int prec, int64_t excl, int rank, int world, bool pre_only = false) {
     const bool self = dTr == nullptr;
     const int64_t L = n + m - 1;
     const size_t eb = elt_bytes(prec);
@@ -293,6 +302,7 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
     pp.nrm32 = (float*)ctx->nrm.p; pp.nrm64 = (double*)ctx->nrm.p;
     if (half) {
         MP_CUDA(ctx, ensure(ctx->scale, (size_t)d * sizeof(double)));
+        MP_CUDA(ctx, ensure(ctx->scale_r, (size_t)d * sizeof(double)));
         MP_CUDA(ctx, ensure(ctx->maxbits, (size_t)d * 2 * sizeof(unsigned long long)));
         MP_CUDA(ctx, ensure(ctx->flat, (size_t)n * d * 3 * 2));
         pp.scale = (double*)ctx->scale.p; pp.maxbits = (unsigned long long*)ctx->maxbits.p; pp.flat = ctx->flat.p;
@@ -307,9 +317,11 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
         MP_CUDA(ctx, ensure(*B[3], (size_t)n * Dp * tb));
         MP_CUDA(ctx, ensure(*B[4], (size_t)L * Dp * tb));
         pp.T = sidx == 0 ? dT : dTr;
+        if (half) pp.scale = (double*)(sidx == 0 ? ctx->scale.p : ctx->scale_r.p);   // one scale per series
         pp.st = B[0]->p; pp.st_pair = B[1]->p; pp.mu = B[2]->p; pp.mup = B[3]->p; pp.tw = B[4]->p;
         MP_CUDA(ctx, mpk::launch_precompute(prec, pp, s));
     }
+    if (pre_only) return MP_OK;   // mp_selftest_seeds
 
     // keys (FP16 / Mixed use the FP32 key format: float bits of the half-precision sum)
     const size_t kb = (size_t)n * d * (prec == MP_FP64 ? 16 : 8);
@@ -334,7 +346,41 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
         mp.n = n; mp.d = (int)d; mp.m = (int)m; mp.H = (int)H;
         mp.seed_kahan = prec == MP_FP16CK ? 1 : 0;
         const int64_t nq = std::max<int64_t>(1, (n + pl.H - 1) / pl.H);
-        return enqueue_tiles(ctx, s, prec, self, mp, pl, bb[rank], bb[rank + 1], 0, nq, true);
+        if (!(tc_seeds(ctx, prec) && var.cta))
+            return enqueue_tiles(ctx, s, prec, self, mp, pl, bb[rank], bb[rank + 1], 0, nq, true);
+        // tensor-core seeds (NEXT-3): per row chunk, one seed GEMM for the chunk's re-seed rows,
+        // then the fused kernel over the chunk's tiles reading the table
+        const int64_t B0 = bb[rank], B1 = bb[rank + 1];
+        if (B1 <= B0) return MP_OK;
+        const int64_t dlo = pl.dlo + B0 * pl.nc, dhi = std::min<int64_t>(pl.dlo + B1 * pl.nc - 1, pl.dhi);
+        const int64_t ncol = n + 8;
+        const int64_t per_seg = std::max<int64_t>(1, pl.H / H) * d * ncol * 2;   // table bytes per row segment
+        const int64_t qs = std::max<int64_t>(1, kSeedTabBytes / per_seg);
+        MP_CUDA(ctx, ensure(ctx->seedtab, (size_t)(qs * per_seg + 64)));
+        mpk::SeedParams sp{};
+        sp.Tq = dT; sp.Tr = self ? dT : dTr;
+        sp.scale_q = (const double*)ctx->scale.p;
+        sp.scale_r = (const double*)(self ? ctx->scale.p : ctx->scale_r.p);
+        sp.mu_q = (const float*)ctx->mu_q.p;
+        sp.mu_r = (const float*)(self ? ctx->mu_q.p : ctx->mu_r.p);
+        sp.tab = ctx->seedtab.p;
+        sp.n = n; sp.d = (int)d; sp.m = (int)m; sp.H = (int)H;
+        MP_CUDA(ctx, cudaEventRecord(ctx->ev0, s));
+        for (int64_t q0 = 0; q0 < nq; q0 += qs) {
+            const int64_t q1 = std::min(nq, q0 + qs), i0 = q0 * pl.H, i1 = std::min(n, q1 * pl.H);
+            sp.r_lo = (i0 + H - 1) / H;
+            sp.r_hi = (i1 + H - 1) / H;
+            sp.j_lo = std::max<int64_t>(0, i0 + dlo) / 8 * 8;
+            sp.j_hi = std::min<int64_t>(n, std::max<int64_t>(0, i1 - 1 + dhi + 1));
+            if (sp.j_hi <= sp.j_lo) continue;
+            sp.ldj = (sp.j_hi - sp.j_lo + 7) / 8 * 8;
+            MP_CUDA(ctx, mpk::launch_seed_gemm(sp, s));
+            mp.seed_tab = sp.tab;
+            mp.tab_r_lo = sp.r_lo; mp.tab_r_hi = sp.r_hi; mp.tab_j_lo = sp.j_lo; mp.tab_ldj = sp.ldj;
+            mp_status st2 = enqueue_tiles(ctx, s, prec, self, mp, pl, B0, B1, q0, q1, false);
+            if (st2 != MP_OK) return st2;
+        }
+        MP_CUDA(ctx, cudaEventRecord(ctx->ev1, s));
     }
     return MP_OK;
 }
@@ -795,6 +841,8 @@ mp_status mp_init(mp_ctx** out, const mp_config* cfg) {
         for (int i = 0; i < 4; ++i) ctx->H[i] = cfg->reseed_h[i];
         ctx->H[4] = cfg->reseed_h[2];  // FP16C follows FP16
         ctx->H[5] = cfg->reseed_h[3];  // FP16CK follows MIXED
+        if (cfg->seed_mode != MP_SEEDS_DIRECT && cfg->seed_mode != MP_SEEDS_TC) { delete ctx; return MP_ERR_INVALID; }
+        ctx->seed_mode = cfg->seed_mode;
     }
     for (int i = 0; i < 6; ++i)
         if (ctx->H[i] < 0 || ctx->H[i] > (int64_t(1) << 30)) { delete ctx; return MP_ERR_INVALID; }
@@ -818,7 +866,8 @@ void mp_free(mp_ctx* ctx) {
     cudaSetDevice(ctx->device);
     Buf* bufs[] = {&ctx->dT, &ctx->dTr, &ctx->st_q, &ctx->st_r, &ctx->tw_q, &ctx->tw_r, &ctx->mu_q,
                    &ctx->mu_r, &ctx->mup_q, &ctx->mup_r, &ctx->nrm, &ctx->keys, &ctx->ext, &ctx->seg, &ctx->counter, &ctx->dP,
-                   &ctx->dI, &ctx->flag, &ctx->stp_q, &ctx->stp_r, &ctx->scale, &ctx->maxbits, &ctx->flat};
+                   &ctx->dI, &ctx->flag, &ctx->stp_q, &ctx->stp_r, &ctx->scale, &ctx->scale_r, &ctx->maxbits, &ctx->flat,
+                   &ctx->seedtab};
     for (Buf* b : bufs) release(*b);
     if (ctx->hflag) cudaFreeHost(ctx->hflag);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
@@ -962,6 +1011,56 @@ mp_status mp_selftest_sort_scan(mp_ctx* ctx, int64_t d, int64_t count, const flo
     release(a);
     release(b);
     return e == cudaSuccess ? MP_OK : cuda_fail(ctx, e, "mp_selftest_sort_scan");
+}
+
+mp_status mp_selftest_seeds(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, int64_t n, int64_t m,
+                            mp_precision prec, int64_t H, int64_t r_lo, int64_t r_hi, double* out,
+                            double* scale_out) {
+    if (!ctx) return MP_ERR_INVALID;
+    mp_status st = validate(ctx, T, d, n, m, prec);
+    if (st != MP_OK) return st;
+    if (!out || !scale_out || (prec != MP_MIXED && prec != MP_FP16CK) || H < 1 || r_lo < 0 || r_hi <= r_lo ||
+        r_hi > (n + H - 1) / H)
+        return fail(ctx, MP_ERR_INVALID, "bad arguments");
+    MP_CUDA(ctx, cudaSetDevice(ctx->device));
+    cudaStream_t s = ctx->stream;
+    const int64_t L = n + m - 1;
+    MP_CUDA(ctx, ensure(ctx->dT, (size_t)d * L * 8));
+    MP_CUDA(ctx, cudaMemcpyAsync(ctx->dT.p, T, (size_t)d * L * 8, cudaMemcpyHostToDevice, s));
+    if (Tr) {
+        MP_CUDA(ctx, ensure(ctx->dTr, (size_t)d * L * 8));
+        MP_CUDA(ctx, cudaMemcpyAsync(ctx->dTr.p, Tr, (size_t)d * L * 8, cudaMemcpyHostToDevice, s));
+    }
+    const double* dT = (const double*)ctx->dT.p;
+    const double* dTr = Tr ? (const double*)ctx->dTr.p : nullptr;
+    st = run_partial(ctx, s, dT, dTr, d, n, m, prec, 0, 0, 1, true);
+    if (st != MP_OK) return st;
+    const bool self = Tr == nullptr;
+    mpk::SeedParams sp{};
+    sp.Tq = dT; sp.Tr = self ? dT : dTr;
+    sp.scale_q = (const double*)ctx->scale.p;
+    sp.scale_r = (const double*)(self ? ctx->scale.p : ctx->scale_r.p);
+    sp.mu_q = (const float*)ctx->mu_q.p;
+    sp.mu_r = (const float*)(self ? ctx->mu_q.p : ctx->mu_r.p);
+    sp.n = n; sp.d = (int)d; sp.m = (int)m; sp.H = (int)H;
+    sp.r_lo = r_lo; sp.r_hi = r_hi; sp.j_lo = 0; sp.j_hi = n; sp.ldj = (n + 7) / 8 * 8;
+    const size_t cnt = (size_t)(r_hi - r_lo) * d * sp.ldj;
+    Buf tb;
+    MP_CUDA(ctx, ensure(tb, cnt * 2));
+    sp.tab = tb.p;
+    std::vector<__half> h(cnt);
+    cudaError_t e = mpk::launch_seed_gemm(sp, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(h.data(), tb.p, cnt * 2, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(scale_out, ctx->scale.p, d * 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess && !self) e = cudaMemcpyAsync(scale_out + d, ctx->scale_r.p, d * 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    release(tb);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "mp_selftest_seeds");
+    for (int64_t r = 0; r < r_hi - r_lo; ++r)       // unpack [r][dim][ldj] half -> [r][dim][n] double
+        for (int64_t k = 0; k < d; ++k)
+            for (int64_t j = 0; j < n; ++j)
+                out[(r * d + k) * n + j] = (double)__half2float(h[(r * d + k) * sp.ldj + j]);
+    return finish_partial(ctx, s);
 }
 
 mp_status mp_selftest_precompute(mp_ctx* ctx, const double* T, int64_t d, int64_t n, int64_t m,

@@ -64,6 +64,36 @@ template <int DL, int G, int NW> struct CtaGeoH {
     static constexpr size_t bytes = col_bytes + row_bytes + stg_bytes + 16;
 };
 
+// Seeds of a cell pair from the tensor-core seed table (MP_SEEDS_TC, mp_seed_tc.cu) when every
+// valid cell of the pair starts on a table row (a re-seed row r H inside the table's row range
+// and column window); returns false otherwise (the caller computes the seeds directly).
+template <int DL, int G>
+__device__ __forceinline__ bool seed_pair_tab(const MainParams& p, int g, long long delta0, bool ok0, bool ok1,
+                                              long long row0, long long row1, __half2 (&QT)[DL]) {
+    if (p.seed_tab == nullptr) return false;
+    const __half* tab = reinterpret_cast<const __half*>(p.seed_tab);
+    const long long row[2] = {row0, row1};
+    const bool ok[2] = {ok0, ok1};
+    long long base[2] = {0, 0};
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+        if (!ok[u]) continue;
+        if (row[u] % p.H != 0) return false;
+        const long long r = row[u] / p.H, j = row[u] + delta0 + u;
+        if (r < p.tab_r_lo || r >= p.tab_r_hi || j < p.tab_j_lo || j >= p.tab_j_lo + p.tab_ldj) return false;
+        base[u] = (r - p.tab_r_lo) * p.d * p.tab_ldj + (j - p.tab_j_lo);
+    }
+#pragma unroll
+    for (int kk = 0; kk < DL; ++kk) {
+        const int dim = kk * G + g;
+        const bool pad = dim >= p.d;
+        const __half h0 = pad ? __float2half(-1.f) : (ok0 ? tab[base[0] + (long long)dim * p.tab_ldj] : __float2half(0.f));
+        const __half h1 = pad ? __float2half(-1.f) : (ok1 ? tab[base[1] + (long long)dim * p.tab_ldj] : __float2half(0.f));
+        QT[kk] = __halves2half2(ok0 ? h0 : __low2half(QT[kk]), ok1 ? h1 : __high2half(QT[kk]));
+    }
+    return true;
+}
+
 template <int DL, int G, int NW, bool SELF, int MODE>
 __global__ void __launch_bounds__(32 * NW, CtaShapeH<G>::MINB)
 mp_diag_cta_h(const MainParams p) {
@@ -189,7 +219,8 @@ mp_diag_cta_h(const MainParams p) {
         __half2 QT[DL];
 #pragma unroll
         for (int kk = 0; kk < DL; ++kk) QT[kk] = __float2half2_rn((kk * G + g) >= d ? -1.f : 0.f);
-        if (lo[0] < hi[0] || lo[1] < hi[1])
+        if ((lo[0] < hi[0] || lo[1] < hi[1]) &&
+            !seed_pair_tab<DL, G>(p, g, dP, lo[0] < hi[0], lo[1] < hi[1], lo[0], lo[1], QT))
             seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, dP, lo[0] < hi[0], lo[1] < hi[1], lo[0], lo[1], QT, p.seed_kahan != 0);
 
         const int nrows = (int)(r1 - r0);
@@ -212,7 +243,8 @@ mp_diag_cta_h(const MainParams p) {
                 to_seed = H;
                 const long long row = R0 + s0;
                 const bool u0 = row > lo[0] && row < hi[0], u1 = row > lo[1] && row < hi[1];
-                if (u0 || u1) seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, dP, u0, u1, row, row, QT, p.seed_kahan != 0);
+                if ((u0 || u1) && !seed_pair_tab<DL, G>(p, g, dP, u0, u1, row, row, QT))
+                    seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, dP, u0, u1, row, row, QT, p.seed_kahan != 0);
                 seeded_step = s0;
             }
             const int nxt = min(s0 + 2 * SB, nrows);

@@ -35,6 +35,27 @@ struct MainParams {
     long long q_lo;               // block-major order: first row segment of the launch's row
                                   // window (0; > 0 only for a streamed chunk, mp_compute_stream)
     int seed_kahan;               // Mixed kernels: 1 -> Kahan-compensated FP32 seeds (MP_FP16CK)
+    // tensor-core seed table (half block kernels, mp_config.seed_mode = MP_SEEDS_TC): seeds of
+    // rows r H, r in [tab_r_lo, tab_r_hi), columns [tab_j_lo, tab_j_lo + tab_ldj) at
+    // seed_tab[((r - tab_r_lo) * d + dim) * tab_ldj + (j - tab_j_lo)]; nullptr: direct seeds
+    const void* seed_tab;
+    long long tab_r_lo, tab_r_hi, tab_j_lo, tab_ldj;
+};
+
+// Tensor-core seed GEMM (mp_seed_tc.cu): seeds of rows r H, r in [r_lo, r_hi), against columns
+// [j_lo, j_hi) for every dimension, from the FP64 input scaled by the per-dimension power of two
+// (reading G16) and the FP32 window means of the Mixed precalc.
+struct SeedParams {
+    const double* Tq;      // query series [dim][L]
+    const double* Tr;      // reference series (== Tq for a self-join)
+    const double* scale_q; // [d]
+    const double* scale_r;
+    const float* mu_q;     // window means [dim][n] (FP32)
+    const float* mu_r;
+    void* tab;             // out (half): [(r - r_lo) * d + dim][ldj]
+    long long n;
+    int d, m, H;
+    long long r_lo, r_hi, j_lo, j_hi, ldj;   // ldj: a multiple of 8, >= j_hi - j_lo
 };
 
 struct PreParams {
@@ -92,6 +113,7 @@ cudaError_t launch_keys_to_ext(int prec, const void* keys, void* ext, long long 
                                cudaStream_t s);
 cudaError_t launch_key_mask(long long count, long long* ext, const long long* gv, cudaStream_t s);
 cudaError_t launch_check_finite(const double* x, long long count, int* flag, cudaStream_t s);
+cudaError_t launch_seed_gemm(const SeedParams& p, cudaStream_t s);
 // stage self-tests (include/mp.h)
 cudaError_t launch_selftest_sort_scan(int d, long long count, const float* in, float* out, cudaStream_t s);
 cudaError_t launch_selftest_unpack(int prec, const void* st, long long n, int d, double* df, double* dg, double* a,

@@ -24,7 +24,8 @@ STATUS = {0: "MP_OK", 1: "MP_ERR_INVALID", 2: "MP_ERR_NOMEM", 3: "MP_ERR_CUDA", 
 EXPORTS = ["mp_init", "mp_free", "mp_last_error", "mp_version", "mp_compute", "mp_compute_device",
            "mp_key_words", "mp_partial_device", "mp_key_mask_device", "mp_finalize_device",
            "mp_plan_bands", "mp_plan_diagonals", "mp_last_timing", "mp_selftest_sort_scan",
-           "mp_selftest_precompute", "mp_compute_stream", "mp_plan_stream", "mp_last_stream_info"]
+           "mp_selftest_precompute", "mp_compute_stream", "mp_plan_stream", "mp_last_stream_info",
+           "mp_selftest_seeds"]
 
 _lib = None
 
@@ -36,7 +37,10 @@ class MPError(RuntimeError):
 
 
 class _Config(ctypes.Structure):
-    _fields_ = [("device", ctypes.c_int), ("reseed_h", ctypes.c_int64 * 4)]
+    _fields_ = [("device", ctypes.c_int), ("reseed_h", ctypes.c_int64 * 4), ("seed_mode", ctypes.c_int)]
+
+
+SEED_MODES = {"direct": 0, "tc": 1}   # mp_config.seed_mode (MP_SEEDS_DIRECT / MP_SEEDS_TC)
 
 
 def load():
@@ -78,6 +82,8 @@ def load():
     lib.mp_selftest_sort_scan.restype = i32
     lib.mp_selftest_precompute.argtypes = [p, p, i64, i64, i64, i32, p, p, p]
     lib.mp_selftest_precompute.restype = i32
+    lib.mp_selftest_seeds.argtypes = [p, p, p, i64, i64, i64, i32, i64, i64, i64, p, p]
+    lib.mp_selftest_seeds.restype = i32
     lib.mp_compute_stream.argtypes = [p, p, p, i64, i64, i64, i32, i64, i64, p, p]
     lib.mp_compute_stream.restype = i32
     lib.mp_plan_stream.argtypes = [i64, i64, i64, i32, i64, i32, i64, i64, p, p]
@@ -164,10 +170,11 @@ def _need(t, name, dtype, device, shape=None, min_numel=None):
 class Context:
     """One context per host thread / GPU (mp_init ... mp_free)."""
 
-    def __init__(self, device: int = 0, reseed_h=None):
+    def __init__(self, device: int = 0, reseed_h=None, seed_mode="direct"):
         lib = load()
         cfg = _Config()
         cfg.device = device
+        cfg.seed_mode = SEED_MODES[seed_mode] if isinstance(seed_mode, str) else int(seed_mode)
         h = list(reseed_h or [0, 0, 0, 0])
         for i in range(4):
             cfg.reseed_h[i] = int(h[i])
@@ -334,6 +341,23 @@ class Context:
                                            *[o.ctypes.data_as(ctypes.c_void_p) for o in outs])
         self._check(st, "mp_selftest_precompute")
         return tuple(outs)
+
+    def selftest_seeds(self, T, m, prec="mixed", H=256, rows=(0, 1), Tr=None):
+        """Tensor-core seed table (MP_SEEDS_TC) of re-seed rows r*H, r in [rows[0], rows[1]), against
+        every column: ((r, d, n) doubles in the precalc's scaled units, per-dimension scales)."""
+        T = np.ascontiguousarray(T, dtype=np.float64)
+        d, L = T.shape
+        n = L - m + 1
+        Tr_ = None if Tr is None else np.ascontiguousarray(Tr, dtype=np.float64)
+        r0, r1 = rows
+        out = np.empty((r1 - r0, d, n))
+        sc = np.zeros(2 * d)
+        st = load().mp_selftest_seeds(self._ctx, T.ctypes.data_as(ctypes.c_void_p),
+                                      None if Tr_ is None else Tr_.ctypes.data_as(ctypes.c_void_p),
+                                      d, n, m, _prec(prec), H, r0, r1, out.ctypes.data_as(ctypes.c_void_p),
+                                      sc.ctypes.data_as(ctypes.c_void_p))
+        self._check(st, "mp_selftest_seeds")
+        return out, (sc[:d] if Tr is None else sc)
 
     def last_timing(self):
         ms = ctypes.c_double()
