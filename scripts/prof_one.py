@@ -20,7 +20,7 @@ T = torch.from_numpy(cfg["T"]).cuda()
 Tr = None if cfg["Tr"] is None else torch.from_numpy(cfg["Tr"]).cuda()
 P = torch.empty(d, n, dtype=torch.float64, device="cuda")
 I = torch.empty(d, n, dtype=torch.int64, device="cuda")
-ctx = mstamp.Context(0)
+ctx = mstamp.Context(0, seed_mode=os.environ.get("MP_SEED_MODE", "direct"))
 import subprocess  # noqa: E402
 for r in range(reps):
     ctx.compute_device(T, m, P, I, prec, e, Tr=Tr)
