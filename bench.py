@@ -408,7 +408,7 @@ def main():
         Tr = None if cfg["Tr"] is None else torch.from_numpy(cfg["Tr"]).to(dev)
         return cfg, T, Tr
 
-    def runner(cfg, T, Tr):
+    def runner(cfg, T, Tr, ctx=ctx):
         d, n, m, e = cfg["d"], cfg["n"], cfg["m"], cfg["exclusion"]
         P = torch.empty(d, n, dtype=torch.float64, device=dev)
         I = torch.empty(d, n, dtype=torch.int64, device=dev)
@@ -503,6 +503,17 @@ def main():
                                   "steps": st}
             per_prec[prec]["alu_frac"] = frac(per_prec[prec]["main_kernel_ms"], d, cells, self_join, prec)
             per_prec[prec]["computed_cell_dims_per_s"] = cells * d / (per_prec[prec]["main_kernel_ms"] * 1e-3)
+        # Mixed with tensor-core seeds (seed_mode MP_SEEDS_TC, NEXT-3): the seed GEMMs run inside
+        # the timed step (main_kernel_ms spans the seed GEMMs and the fused-kernel chunks)
+        if d >= 64:
+            ctx_tc = mstamp.Context(local, seed_mode="tc")
+            timed_tc, _, _ = runner(cfg, T, Tr, ctx_tc)
+            p_ms, p_kms, _ = timed_tc("mixed", max(1, min(args.steps, 3)), 1)
+            per_prec["mixed_tc_seeds"] = {"value": dn2 / (p_ms * 1e-3), "ms_per_step": p_ms, "main_kernel_ms": p_kms,
+                                          "steps": max(1, min(args.steps, 3)),
+                                          "alu_frac": frac(p_kms, d, cells, self_join, "mixed")}
+            ctx_tc.close()
+            del timed_tc
 
     context = None
     if not args.no_context and world == 1 and args.config != "C2":

@@ -1,0 +1,9 @@
+// Explicit instantiations of the half2 fused diagonal kernel (FP16 / Mixed / FP16C).
+#define MP_DIAG_IMPL
+#include "mp_diag16.cuh"
+namespace mpk {
+template struct InstH<1, 1, false, 3>;
+template struct InstH<2, 1, false, 3>;
+template struct InstH<4, 1, false, 3>;
+template struct InstH<8, 1, false, 3>;
+}  // namespace mpk

@@ -252,7 +252,9 @@ mp_status enqueue_tiles(mp_ctx* ctx, cudaStream_t s, int prec, bool self, mpk::M
 }
 
 // Tensor-core seeds apply to the FP32-precalc half modes (Mixed, FP16CK) on the block kernels.
-constexpr int64_t kSeedTabBytes = int64_t(1) << 30;   // seed table per row chunk (device bytes)
+// seed table per row chunk (device bytes): up to 128 seed rows (one MMA tile of M = 128) per chunk,
+// so each Hankel operand tile the GEMM builds serves as many rows as fit
+constexpr int64_t kSeedTabBytes = int64_t(8) << 30;
 bool tc_seeds(const mp_ctx* ctx, int prec) {
     return ctx->seed_mode == MP_SEEDS_TC && (prec == MP_MIXED || prec == MP_FP16CK);
 }
@@ -344,7 +346,6 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
         mp.mu_r = self ? ctx->mup_q.p : ctx->mup_r.p;
         mp.keys = ctx->keys.p;
         mp.n = n; mp.d = (int)d; mp.m = (int)m; mp.H = (int)H;
-        mp.seed_kahan = prec == MP_FP16CK ? 1 : 0;
         const int64_t nq = std::max<int64_t>(1, (n + pl.H - 1) / pl.H);
         if (!(tc_seeds(ctx, prec) && var.cta))
             return enqueue_tiles(ctx, s, prec, self, mp, pl, bb[rank], bb[rank + 1], 0, nq, true);
@@ -354,8 +355,9 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
         if (B1 <= B0) return MP_OK;
         const int64_t dlo = pl.dlo + B0 * pl.nc, dhi = std::min<int64_t>(pl.dlo + B1 * pl.nc - 1, pl.dhi);
         const int64_t ncol = n + 8;
-        const int64_t per_seg = std::max<int64_t>(1, pl.H / H) * d * ncol * 2;   // table bytes per row segment
-        const int64_t qs = std::max<int64_t>(1, kSeedTabBytes / per_seg);
+        const int64_t rows_seg = std::max<int64_t>(1, pl.H / H);              // seed rows per row segment
+        const int64_t per_seg = rows_seg * d * ncol * 2;                       // table bytes per row segment
+        const int64_t qs = std::max<int64_t>(1, std::min(kSeedTabBytes / per_seg, std::max<int64_t>(1, 128 / rows_seg)));
         MP_CUDA(ctx, ensure(ctx->seedtab, (size_t)(qs * per_seg + 64)));
         mpk::SeedParams sp{};
         sp.Tq = dT; sp.Tr = self ? dT : dTr;
@@ -765,7 +767,6 @@ mp_status run_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, 
     mp.mu_r = rs.mup.ptr();
     mp.keys = S.sq.keys.ptr();
     mp.n = n; mp.d = (int)d; mp.m = (int)m; mp.H = (int)H;
-    mp.seed_kahan = prec == MP_FP16CK ? 1 : 0;
 
     ctx->last_launches = 0;
     ctx->last_ms = 0.0;

@@ -108,15 +108,19 @@ __device__ __forceinline__ void ldv(const T* __restrict__ rowp, int g, T (&out)[
 
 // Seeds of one cell pair (diagonals delta0, delta0 + 1): direct centred dot products
 // (reading G8) at rows row0 / row1 (cells with ok_u false keep their QT).
-// Mixed -> FP32 operands and accumulation rounded to half (the FP32 precalc; kh: with Kahan
-// compensation, MP_FP16CK, the text's FP16C reading L786-791); FP16 -> half arithmetic;
+// Mixed -> FP32 operands and accumulation rounded to half (the FP32 precalc; FP16CK: with Kahan
+// compensation, the text's FP16C reading L786-791); FP16 -> half arithmetic;
 // FP16C -> half arithmetic with Kahan compensation (Fig. 1 reading).  When both cells start on the
 // same row the row window is shared and the second column window is the first shifted by one.
+// Half-kernel modes: 0 FP16, 1 Mixed, 2 FP16C (Fig. 1), 3 FP16CK (the text's FP16C: Mixed with
+// Kahan-compensated FP32 seeds), 5 Mixed / FP16CK reading the tensor-core seed table (block kernel)
+constexpr bool fp32_precalc(int mode) { return mode == 1 || mode == 3 || mode == 5; }
+
 template <int DL, int G, int MODE, class TS>
 __device__ __forceinline__ void seed_pair_h(const TS* __restrict__ tw_q, const TS* __restrict__ tw_r,
                                             const TS* __restrict__ mu_q, const TS* __restrict__ mu_r,
                                             int m, int d, int g, long long delta0, bool ok0, bool ok1,
-                                            long long row0, long long row1, __half2 (&QT)[DL], bool kh) {
+                                            long long row0, long long row1, __half2 (&QT)[DL]) {
     constexpr int D = DL * G;
     const long long delta[2] = {delta0, delta0 + 1};
     using TA = TS;
@@ -124,9 +128,9 @@ __device__ __forceinline__ void seed_pair_h(const TS* __restrict__ tw_q, const T
     TA acc0[DL], acc1[DL];
 #pragma unroll
     for (int kk = 0; kk < DL; ++kk) { acc0[kk] = (TA)0.f; acc1[kk] = (TA)0.f; }
-    const bool comp = MODE == 2 || (MODE == 1 && kh);
-    auto kadd = [comp](TA& acc, TA& cp, TA v) {
-        if (comp) {  // compensated accumulation (warp-uniform: a launch parameter)
+    constexpr bool comp = MODE == 2 || MODE == 3;
+    auto kadd = [](TA& acc, TA& cp, TA v) {
+        if constexpr (comp) {  // compensated accumulation
             const TA y = v - cp;
             const TA t2 = acc + y;
             cp = (t2 - acc) - y;
@@ -204,7 +208,7 @@ __device__ __forceinline__ void seed_pair_h(const TS* __restrict__ tw_q, const T
 template <int DL, int G, bool SELF, int MODE>
 __global__ void __launch_bounds__(128)
 mp_diag_h(const MainParams p) {
-    constexpr bool MIXED = MODE == 1;
+    constexpr bool MIXED = fp32_precalc(MODE);
     using Gm = Geo<G, 2>;
     using SM = SmemH<DL, G>;
     using TS = typename std::conditional<MIXED, float, __half>::type;  // seed operand type
@@ -327,7 +331,7 @@ mp_diag_h(const MainParams p) {
 
         __half2 QT[DL];
         auto seed_pair = [&](bool ok0, bool ok1, long long row0, long long row1) {
-            seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, delta[0], ok0, ok1, row0, row1, QT, p.seed_kahan != 0);
+            seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, delta[0], ok0, ok1, row0, row1, QT);
         };
 #pragma unroll
         for (int kk = 0; kk < DL; ++kk) QT[kk] = __float2half2_rn((kk * G + g) >= d ? -1.f : 0.f);

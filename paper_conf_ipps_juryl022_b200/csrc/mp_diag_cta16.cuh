@@ -99,7 +99,7 @@ __global__ void __launch_bounds__(32 * NW, CtaShapeH<G>::MINB)
 mp_diag_cta_h(const MainParams p) {
     using Cg = CtaGeoH<DL, G, NW>;
     using K = unsigned long long;
-    using TS = typename std::conditional<MODE == 1, float, __half>::type;  // seed operand type
+    using TS = typename std::conditional<fp32_precalc(MODE), float, __half>::type;  // seed operand type
     constexpr int D = Cg::D, NP = Cg::NP, NCC = Cg::NCC, RR = Cg::RR, RC = Cg::RC, SB = Cg::SB, NT = Cg::NT;
     static_assert(NP * G == NT, "G must divide the block");
 
@@ -219,9 +219,14 @@ mp_diag_cta_h(const MainParams p) {
         __half2 QT[DL];
 #pragma unroll
         for (int kk = 0; kk < DL; ++kk) QT[kk] = __float2half2_rn((kk * G + g) >= d ? -1.f : 0.f);
-        if ((lo[0] < hi[0] || lo[1] < hi[1]) &&
-            !seed_pair_tab<DL, G>(p, g, dP, lo[0] < hi[0], lo[1] < hi[1], lo[0], lo[1], QT))
-            seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, dP, lo[0] < hi[0], lo[1] < hi[1], lo[0], lo[1], QT, p.seed_kahan != 0);
+        // seeds: the tensor-core table (MP_SEEDS_TC) or direct dot products (FP16CK: compensated)
+        // seeds: the tensor-core table (MODE 5) where the cell starts on a table row, else direct
+        auto seed = [&](bool u0, bool u1, long long row0, long long row1) {
+            if constexpr (MODE == 5)
+                if (seed_pair_tab<DL, G>(p, g, dP, u0, u1, row0, row1, QT)) return;
+            seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, dP, u0, u1, row0, row1, QT);
+        };
+        if (lo[0] < hi[0] || lo[1] < hi[1]) seed(lo[0] < hi[0], lo[1] < hi[1], lo[0], lo[1]);
 
         const int nrows = (int)(r1 - r0);
         const int R0 = (int)r0, C0 = (int)(r0 + delta0);  // row / first column of step 0
@@ -243,8 +248,7 @@ mp_diag_cta_h(const MainParams p) {
                 to_seed = H;
                 const long long row = R0 + s0;
                 const bool u0 = row > lo[0] && row < hi[0], u1 = row > lo[1] && row < hi[1];
-                if ((u0 || u1) && !seed_pair_tab<DL, G>(p, g, dP, u0, u1, row, row, QT))
-                    seed_pair_h<DL, G, MODE, TS>(tw_q, tw_r, mu_q, mu_r, m, d, g, dP, u0, u1, row, row, QT, p.seed_kahan != 0);
+                if (u0 || u1) seed(u0, u1, row, row);
                 seeded_step = s0;
             }
             const int nxt = min(s0 + 2 * SB, nrows);

@@ -34,7 +34,6 @@ struct MainParams {
     long long delta_lo, delta_hi; // diagonal range [lo, hi] (j = i + delta)
     long long q_lo;               // block-major order: first row segment of the launch's row
                                   // window (0; > 0 only for a streamed chunk, mp_compute_stream)
-    int seed_kahan;               // Mixed kernels: 1 -> Kahan-compensated FP32 seeds (MP_FP16CK)
     // tensor-core seed table (half block kernels, mp_config.seed_mode = MP_SEEDS_TC): seeds of
     // rows r H, r in [tab_r_lo, tab_r_hi), columns [tab_j_lo, tab_j_lo + tab_ldj) at
     // seed_tab[((r - tab_r_lo) * d + dim) * tab_ldj + (j - tab_j_lo)]; nullptr: direct seeds

@@ -8,6 +8,10 @@
 #include "mp_diag_cta64.cuh"
 #include "mp_diag_ctab.cuh"
 
+#ifndef MP_MIX_STATS_KAHAN
+#define MP_MIX_STATS_KAHAN 0   // Mixed window statistics with Kahan sums (1: experiment; FP16CK has them)
+#endif
+
 namespace mpk {
 
 // ------------------------------------------------------------------ precompute
@@ -85,7 +89,7 @@ __global__ void pre_pm(const PreParams p) {
     T* tw = reinterpret_cast<T*>(p.tw);
     T* mup = reinterpret_cast<T*>(p.mup);
     // pm_G > 0: dim kk*G + g is stored at g*DL + kk (each lane's dims contiguous)
-    const long long o = p.pm_G > 0 ? t * Dp + (dim % p.pm_G) * p.pm_DL + dim / p.pm_G : gid;
+    const long long o = p.pm_G > 0 ? t * Dp + (dim % p.pm_G) * p.pm_DL + dim / p.pm_G : t * Dp + dim;
     tw[o] = dim < d ? (T)p.T[(long long)dim * p.T_ld + (t - p.T_off)] : (T)0;
     if (t < p.w1) mup[o] = dim < d ? (T)reinterpret_cast<const A*>(p.mu)[(long long)dim * p.s_ld + (t - p.s_off)] : (T)0;
 }
@@ -511,13 +515,17 @@ static long long dispatch_cta64(int op, int G, const MainParams* p, int grid, cu
 }
 
 static long long dispatch(int op, int prec, bool self, int d, const MainParams* p, int grid, cudaStream_t s) {
-    if (prec == P16CK) prec = PMIX;   // the Mixed kernels; the seed compensation is MainParams::seed_kahan
     const Variant v = pick_variant(prec, d);
-    if (v.cta && (prec == P16 || prec == PMIX || prec == P16C)) {
-        const int md = prec == P16 ? 0 : prec == PMIX ? 1 : 2;
+    if (v.cta && (prec == P16 || prec == PMIX || prec == P16C || prec == P16CK)) {
+        // half-kernel modes (mp_diag16.cuh): FP16CK = Mixed with compensated seeds (3); a launch
+        // with a tensor-core seed table (MainParams::seed_tab) takes the table kernel (5)
+        const bool tab = p && p->seed_tab && (prec == PMIX || prec == P16CK);
+        const int md = tab ? 5 : prec == P16 ? 0 : prec == PMIX ? 1 : prec == P16C ? 2 : 3;
         if (md == 0) return self ? dispatch_ctah<true, 0>(op, v.G, p, grid, s) : dispatch_ctah<false, 0>(op, v.G, p, grid, s);
         if (md == 1) return self ? dispatch_ctah<true, 1>(op, v.G, p, grid, s) : dispatch_ctah<false, 1>(op, v.G, p, grid, s);
-        return self ? dispatch_ctah<true, 2>(op, v.G, p, grid, s) : dispatch_ctah<false, 2>(op, v.G, p, grid, s);
+        if (md == 2) return self ? dispatch_ctah<true, 2>(op, v.G, p, grid, s) : dispatch_ctah<false, 2>(op, v.G, p, grid, s);
+        if (md == 3) return self ? dispatch_ctah<true, 3>(op, v.G, p, grid, s) : dispatch_ctah<false, 3>(op, v.G, p, grid, s);
+        return self ? dispatch_ctah<true, 5>(op, v.G, p, grid, s) : dispatch_ctah<false, 5>(op, v.G, p, grid, s);
     }
     if (v.cta && prec == P64) return self ? dispatch_cta64<true>(op, v.G, p, grid, s) : dispatch_cta64<false>(op, v.G, p, grid, s);
     if (v.ctab) return self ? dispatch_ctab<true>(op, v.DL * v.G, p, grid, s) : dispatch_ctab<false>(op, v.DL * v.G, p, grid, s);
@@ -525,6 +533,7 @@ static long long dispatch(int op, int prec, bool self, int d, const MainParams* 
     if (prec == P16) return self ? dispatch_h<true, 0>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 0>(op, v.DL, v.G, p, grid, s);
     if (prec == PMIX) return self ? dispatch_h<true, 1>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 1>(op, v.DL, v.G, p, grid, s);
     if (prec == P16C) return self ? dispatch_h<true, 2>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 2>(op, v.DL, v.G, p, grid, s);
+    if (prec == P16CK) return self ? dispatch_h<true, 3>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 3>(op, v.DL, v.G, p, grid, s);
     if (prec == P64) return self ? dispatch_64f<true>(op, v.DL, v.G, p, grid, s) : dispatch_64f<false>(op, v.DL, v.G, p, grid, s);
     if (prec == P32) return self ? dispatch_t<float, true>(op, v.DL, v.G, v.W, p, grid, s) : dispatch_t<float, false>(op, v.DL, v.G, v.W, p, grid, s);
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
@@ -574,7 +583,7 @@ cudaError_t launch_precompute(int prec, const PreParams& p, cudaStream_t s, bool
             pre_diff_h<float><<<grid1d(cf, 256), 256, 0, s>>>(p);
             pre_pm_h<float><<<grid1d(cpm, 256), 256, 0, s>>>(p);
         } else if (prec == PMIX) {
-            pre_stats_h<float><<<grid1d(cs, 256), 256, 0, s>>>(p);
+            pre_stats_h<float, MP_MIX_STATS_KAHAN><<<grid1d(cs, 256), 256, 0, s>>>(p);
             pre_diff_h<float><<<grid1d(cf, 256), 256, 0, s>>>(p);
             pre_pm_h<float><<<grid1d(cpm, 256), 256, 0, s>>>(p);
         } else if (prec == P16C) {

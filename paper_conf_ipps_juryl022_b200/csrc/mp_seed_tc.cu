@@ -49,7 +49,9 @@ __device__ __forceinline__ void mbar_init(unsigned long long* bar, unsigned coun
 }
 __device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned parity) {
     unsigned ok = 0;
+    long long spins = 0;
     while (!ok) {
+        if (++spins > (1ll << 32)) __trap();   // a lost MMA completion: fail loudly instead of hanging
         asm volatile(
             "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
             : "=r"(ok)

@@ -82,14 +82,16 @@ def load():
     lib.mp_selftest_sort_scan.restype = i32
     lib.mp_selftest_precompute.argtypes = [p, p, i64, i64, i64, i32, p, p, p]
     lib.mp_selftest_precompute.restype = i32
-    lib.mp_selftest_seeds.argtypes = [p, p, p, i64, i64, i64, i32, i64, i64, i64, p, p]
-    lib.mp_selftest_seeds.restype = i32
-    lib.mp_compute_stream.argtypes = [p, p, p, i64, i64, i64, i32, i64, i64, p, p]
-    lib.mp_compute_stream.restype = i32
-    lib.mp_plan_stream.argtypes = [i64, i64, i64, i32, i64, i32, i64, i64, p, p]
-    lib.mp_plan_stream.restype = i32
-    lib.mp_last_stream_info.argtypes = [p, p, p, p, p]
-    lib.mp_last_stream_info.restype = i32
+    optional = {  # absent from libraries built before round 2 (MP_LIB_PATH variants)
+        "mp_selftest_seeds": [p, p, p, i64, i64, i64, i32, i64, i64, i64, p, p],
+        "mp_compute_stream": [p, p, p, i64, i64, i64, i32, i64, i64, p, p],
+        "mp_plan_stream": [i64, i64, i64, i32, i64, i32, i64, i64, p, p],
+        "mp_last_stream_info": [p, p, p, p, p],
+    }
+    for name, args in optional.items():
+        if hasattr(lib, name):
+            getattr(lib, name).argtypes = args
+            getattr(lib, name).restype = i32
     _lib = lib
     return lib
 
