@@ -14,6 +14,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
@@ -578,6 +579,11 @@ struct Side {
     } while (0)
 
 struct Streamer {
+    // MP_STREAM_PROFILE=1: host seconds per phase, printed to stderr at the end of the call
+    double t_sync = 0, t_remap = 0, t_pre = 0, t_fin = 0;
+    static double now() {
+        return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
+    }
     mp_ctx* ctx;
     cudaStream_t s;
     Vmm vm;
@@ -601,6 +607,8 @@ struct Streamer {
         return nm;
     }
     mp_status remap(VArr& a, const std::vector<char>& nm, bool is_keys, int64_t final_upto) {
+        const double t0 = now();
+        struct Acc { double& t; double t0; ~Acc() { t += now() - t0; } } acc{t_remap, t0};
         if (is_keys) {   // save the key granules about to be unmapped (those still accumulating)
             bool any = false;
             for (size_t gi = 0; gi < a.h.size(); ++gi) {
@@ -627,6 +635,7 @@ struct Streamer {
     }
     // precompute positions [a, b) of one series (statistics, pair format, seed operands)
     mp_status precompute(Side& sd, int64_t a, int64_t b) {
+        struct Acc { double& t; double t0; ~Acc() { t += now() - t0; } } acc{t_pre, now()};
         mpk::PreParams pp{};
         pp.n = n; pp.d = (int)d; pp.m = (int)m; pp.Dp = g.Dp;
         const mpk::Variant var = mpk::pick_variant(prec, (int)d);
@@ -782,7 +791,9 @@ mp_status run_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, 
             const int64_t ra = std::max(i0, -dhi), rb = std::min(i1, n - dlo);   // rows with cells
             if (ra >= rb) continue;
             const Ivl rows{i0, i1}, cols{std::max<int64_t>(0, ra + dlo), std::min<int64_t>(n, rb - 1 + dhi + 1)};
-            MP_CUDA(ctx, cudaStreamSynchronize(s));   // the previous launch is done with the windows
+            { const double t0 = Streamer::now();
+              MP_CUDA(ctx, cudaStreamSynchronize(s));   // the previous launch is done with the windows
+              S.t_sync += Streamer::now() - t0; }
             if (self) {
                 const std::vector<Ivl> both{rows, cols};
                 if ((st = S.ensure_side(S.sq, both, &both, i0)) != MP_OK) return st;
@@ -807,11 +818,16 @@ mp_status run_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, 
         if ((st = S.remap(S.sq.keys, S.need_mask(S.sq.keys, {{i0, i1}}, (double)d * g.kb, 0), true, i0)) != MP_OK)
             return st;
         const int64_t w = i1 - i0;
+        const double tf0 = Streamer::now();
         MP_CUDA(ctx, mpk::launch_finalize_window(prec, S.sq.keys.ptr(), i0, i1, (int)d, (double*)S.dPw.p,
                                                  (long long*)S.dIw.p, s));
         MP_CUDA(ctx, cudaMemcpy2DAsync(P + i0, n * 8, S.dPw.p, w * 8, w * 8, d, cudaMemcpyDeviceToHost, s));
         MP_CUDA(ctx, cudaMemcpy2DAsync(I + i0, n * 8, S.dIw.p, w * 8, w * 8, d, cudaMemcpyDeviceToHost, s));
+        S.t_fin += Streamer::now() - tf0;
     }
+    if (std::getenv("MP_STREAM_PROFILE"))
+        std::fprintf(stderr, "mp_compute_stream: host s sync %.3f remap %.3f precompute %.3f finalize %.3f\n", S.t_sync,
+                     S.t_remap, S.t_pre, S.t_fin);
     MP_CUDA(ctx, cudaStreamSynchronize(s));
     double tot = 0;
     for (size_t k = 0; k + 1 < evs.size(); k += 2) {

@@ -43,6 +43,9 @@
 #ifndef MP_CTAB_PAIR
 #define MP_CTAB_PAIR 1      // G == 2: the pair-mode merge (pair_si)
 #endif
+#ifndef MP_CTAB_SIGN
+#define MP_CTAB_SIGN 1      // G == 4: sign-split cross-lane merge (two of three cross-lane steps uniform)
+#endif
 #ifndef MP_CTAB_TA
 #define MP_CTAB_TA 1        // thresholds in rank-contiguous per-slot arrays (read as vectors after
                             // the scan) instead of the stats' 4th word (kept live through the sort)
@@ -134,6 +137,71 @@ template <int DL> __device__ __forceinline__ int pair_pos_of_si(int si) {
     return si < DL ? si : (si == 2 * DL - 1 ? 2 * DL - 1 : 3 * DL - 2 - si);
 }
 
+// Sign-split merge (G == 4, MP_CTAB_SIGN).  Lanes 2 and 3 of a cell hold their distances negated
+// (stored value = sigma_g x true value, sigma = (+, +, -, -)).  A cross-lane compare between lanes of
+// opposite sign is then the same instruction in both lanes, own = min(own, -partner): the positive
+// lane keeps the true minimum, the negative lane the true maximum (negated) -- one FMNMX with a
+// negated operand instead of a lane-dependent min / max pair (FMNMX + predicated FMNMX).  The
+// 64-element merge of four sorted 16-runs: (1) lanes g ^ 2, same register: uniform; in-lane
+// half-cleaners; (2) lanes g ^ 3, same register: uniform; (3) lanes g ^ 1, mirrored register
+// (same-sign pairs: lane-dependent); in-lane half-cleaners (the last layer fused into pair_scan).
+// Result (checked exhaustively against a sort in the stage self-test): lane 0 holds true ranks
+// 0..15 ascending, lane 1 16..31, lane 2 ranks 47 - k at register k, lane 3 ranks 63 - k, all as
+// stored values ascending.  Derived by searching the uniform-step sequences.
+template <int DL> __device__ __forceinline__ void sign_merge4(float (&v)[DL], int g) {
+    static_assert((DL & (DL - 1)) == 0 && DL >= 4, "power-of-two DL");
+#pragma unroll
+    for (int kk = 0; kk < DL; ++kk) v[kk] = fminf(v[kk], -__shfl_xor_sync(FULL, v[kk], 2));
+#pragma unroll
+    for (int dist = DL / 2; dist >= 1; dist >>= 1)
+#pragma unroll
+        for (int kk = 0; kk < DL; ++kk)
+            if ((kk & dist) == 0) cswap(v[kk], v[kk + dist]);
+#pragma unroll
+    for (int kk = 0; kk < DL; ++kk) v[kk] = fminf(v[kk], -__shfl_xor_sync(FULL, v[kk], 3));
+    const bool keep_min = g == 0 || g == 3;   // stored minimum: lanes 0 (+, true min) and 3 (-, true max)
+#pragma unroll
+    for (int kk = 0; kk < DL / 2; ++kk) {
+        const float y1 = __shfl_xor_sync(FULL, v[DL - 1 - kk], 1);
+        const float y2 = __shfl_xor_sync(FULL, v[kk], 1);
+        v[kk] = keep_min ? fminf(v[kk], y1) : fmaxf(v[kk], y1);
+        v[DL - 1 - kk] = keep_min ? fminf(v[DL - 1 - kk], y2) : fmaxf(v[DL - 1 - kk], y2);
+    }
+#pragma unroll
+    for (int dist = DL / 2; dist >= 2; dist >>= 1)
+#pragma unroll
+        for (int kk = 0; kk < DL; ++kk)
+            if ((kk & dist) == 0) cswap(v[kk], v[kk + dist]);
+}
+// true rank held at register kk of lane g after sign_merge4
+template <int DL> __device__ __forceinline__ int sign_rank(int g, int kk) {
+    return g < 2 ? g * DL + kk : (kk == DL - 1 ? (g + 1) * DL - 1 : (g + 1) * DL - 2 - kk);
+}
+// position of rank r in a lane-blocked threshold array read by register (sign_rank inverse)
+template <int DL> __device__ __forceinline__ int sign_pos(int r) {
+    const int b = r / DL, i = r - b * DL;
+    return b < 2 ? r : b * DL + (i == DL - 1 ? DL - 1 : DL - 2 - i);
+}
+// after pair_scan of the stored values (inclusive prefix P_k in register k): the true prefix sums
+// S at the ranks sign_rank(g, k).  t_g = sigma_g P_{DL-1} is the lane's true total; c_g = sum of
+// the totals of the lanes holding lower ranks (positive lanes) or of lanes up to g (negative lanes,
+// whose register k < DL - 1 then holds c_g + P_k = S at rank (g + 1) DL - 2 - k, and the last
+// register the lane's end S = c_g).
+template <int DL> __device__ __forceinline__ void sign_offsets(float (&v)[DL], int g) {
+    const float pos = g < 2 ? 1.f : 0.f;
+    const float t = (g < 2) ? v[DL - 1] : -v[DL - 1];
+    float incl = t;
+#pragma unroll
+    for (int dd = 1; dd < 4; dd <<= 1) {
+        const float y = __shfl_up_sync(FULL, incl, dd, 4);
+        if (g >= dd) incl += y;
+    }
+    const float c = fmaf(-pos, t, incl);   // positive lanes: exclusive prefix; negative: inclusive
+#pragma unroll
+    for (int kk = 0; kk < DL - 1; ++kk) v[kk] += c;
+    v[DL - 1] = fmaf(pos, v[DL - 1], c);
+}
+
 template <int DL, int G, int NT, bool SELF>
 __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32) mp_diag_ctab(const MainParams p) {
     using Cg = CtabGeo<DL, G, NT>;
@@ -142,6 +210,7 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
     constexpr int D = Cg::D, NCC = Cg::NCC, RR = Cg::RR, RC = Cg::RC, SS = Cg::SS, SB = Cg::SB;
     constexpr int NTHR = Cg::NTHR;
     constexpr bool PM = MP_CTAB_PAIR && MP_CTAB_TA && G == 2;   // pair mode (pair_si)
+    constexpr bool SM = MP_CTAB_SIGN && MP_CTAB_TA && G == 4;    // sign-split merge (sign_merge4)
     constexpr int FOLD = SB > MP_FOLD ? SB : MP_FOLD;
 
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -168,7 +237,8 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
     const unsigned stat_bytes = (unsigned)d * 16u;
     const int npad = D - d;
     // padded planes: pair mode D = 0 (a = 1, QT = 2m; sorts first), else D ~ 1e18 (sorts last)
-    const float pad_a = PM ? 1.f : PT<float>::pad_a();
+    constexpr bool ZP = PM || SM;   // padded dims have D = 0 exactly (sort first; ranks shift by npad)
+    const float pad_a = ZP ? 1.f : PT<float>::pad_a();
 
     // padded planes [d, D) never change (TMA writes planes [0, d) of a slot): set them once
     for (int e = tid; e < (RR + RC) * (D - d); e += NT) {
@@ -225,9 +295,9 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
         const bool is_row = pi < nr;
         const int pos = is_row ? R0 + r_lo + pi : C0 + c_lo + (pi - nr);
         const int slot = is_row ? rslot(pos) : RR + cslot(pos);
-        if (MP_CTAB_TA) dst = (int)(Cg::stat_ring_bytes / 4) + slot * D + (PM ? pair_pos_of_si<DL>(q) : q);
+        if (MP_CTAB_TA) dst = (int)(Cg::stat_ring_bytes / 4) + slot * D + (PM ? pair_pos_of_si<DL>(q) : SM ? sign_pos<DL>(q) : q);
         else dst = (slot * SS + plane_of_rank<DL, G>(q)) * 4 + 3;
-        const int r = PM ? q - npad : q;
+        const int r = ZP ? q - npad : q;
         if (r < 0 || r >= d || pos < 0 || pos >= n32) return NINF;
         return __uint_as_float(__ldcg(reinterpret_cast<const unsigned*>(keys + (size_t)pos * d + r) + 1));
     };
@@ -289,7 +359,7 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
 #pragma unroll
                 for (int kk = 0; kk < SC; ++kk) {  // lane g's register c0 + kk is dim (c0 + kk) G + g
                     const bool pad = ((c0 + kk) * G + g) >= d;
-                    QT[c0 + kk] = pad ? (PM ? two_m : -1.f) : acc[kk];
+                    QT[c0 + kk] = pad ? (ZP ? two_m : -1.f) : acc[kk];
                     QL[c0 + kk] = pad ? 0.f : -cmp[kk];
                 }
             }
@@ -298,7 +368,7 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
             seed_cell(lo);
         } else {
 #pragma unroll
-            for (int kk = 0; kk < DL; ++kk) { QT[kk] = (kk * G + g) >= d ? (PM ? two_m : -1.f) : 0.f; QL[kk] = 0.f; }
+            for (int kk = 0; kk < DL; ++kk) { QT[kk] = (kk * G + g) >= d ? (ZP ? two_m : -1.f) : 0.f; QL[kk] = 0.f; }
         }
 
         // first batch landed: patch its thresholds directly (once per tile)
@@ -375,6 +445,11 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
                     // lane holds at register kk after the sort (one test covers row and column)
                     if constexpr (!MP_CTAB_TA) thr[kk] = SELF ? fmaxf(R.w, C.w) : R.w;
                 }
+                if constexpr (SM) {
+                    const float sgn = g < 2 ? 1.f : -1.f;
+#pragma unroll
+                    for (int kk = 0; kk < DL; ++kk) S[kk] *= sgn;
+                }
                 if constexpr (PM) {
                     const float sgn = g ? -1.f : 1.f;
 #pragma unroll
@@ -396,11 +471,15 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
 #pragma unroll
                     for (int kk = 0; kk < DL - 1; ++kk) S[kk] += cg;
                     S[DL - 1] = g ? cg : tot;
+                } else if constexpr (SM) {
+                    sign_merge4<DL>(S, g);
+                    pair_scan<float, DL>(S);                                             // Eq. (2) scan
+                    sign_offsets<DL>(S, g);
                 } else {
                 if constexpr (G > 1) lane_merge<float, DL, G, true>(S, g);
                 pair_scan<float, DL>(S);                                                 // Eq. (2) scan
                 }
-                if constexpr (G > 1 && !PM) {
+                if constexpr (G > 1 && !PM && !SM) {
                     float tot = S[DL - 1];
 #pragma unroll
                     for (int dd = 1; dd < G; dd <<= 1) {
@@ -432,7 +511,7 @@ __global__ void __launch_bounds__(NT, DL <= 16 ? MP_CTAB_MINB16 : MP_CTAB_MINB32
 #pragma unroll
                     for (int kk = 0; kk < DL; ++kk) {
                         const float v = S[kk];
-                        const int pl = kk * G + g, rk = PM ? pair_si<DL>(g, kk) - npad : g * DL + kk;
+                        const int pl = kk * G + g, rk = PM ? pair_si<DL>(g, kk) - npad : SM ? sign_rank<DL>(g, kk) - npad : g * DL + kk;
                         const unsigned vb = __float_as_uint(v);
                         float* rw = MP_CTAB_TA ? TRs + kk : const_cast<float*>(&Rs[pl].w);
                         if (v <= *reinterpret_cast<volatile float*>(rw)) {

@@ -645,10 +645,12 @@ __global__ void selftest_sort_scan(int d, long long count, const float* in, floa
     const bool ok = cell < count;   // whole warps stay converged for the shuffles
     (void)CPW;
     float S[DL];
+    // padded dims sort last (D ~ 1e18), or first with D = 0 in the sign-split merge (ranks shift)
+    constexpr bool SIGN = CTAB && MP_CTAB_SIGN && G == 4;
 #pragma unroll
     for (int kk = 0; kk < DL; ++kk) {
         const int dim = kk * G + g;
-        S[kk] = (ok && dim < d) ? in[cell * d + dim] : PT<float>::pad_a();   // padded dims sort last
+        S[kk] = (ok && dim < d) ? in[cell * d + dim] : (SIGN ? 0.f : PT<float>::pad_a());
     }
     if constexpr (G == 1 && DL >= 8 && last_layer_adjacent<DL>()) {
         sort_scan_fused<float, DL>(S);        // mp_diag, one lane per cell
@@ -657,6 +659,20 @@ __global__ void selftest_sort_scan(int d, long long count, const float* in, floa
 #pragma unroll
         for (int kk = 1; kk < DL; ++kk) S[kk] += S[kk - 1];
     } else {
+        if constexpr (CTAB && MP_CTAB_SIGN && G == 4) {   // mp_diag_ctab, sign-split merge
+#pragma unroll
+            for (int kk = 0; kk < DL; ++kk) S[kk] *= (g < 2 ? 1.f : -1.f);
+            sort_net<float, DL>(S);
+            sign_merge4<DL>(S, g);
+            pair_scan<float, DL>(S);
+            sign_offsets<DL>(S, g);
+#pragma unroll
+            for (int kk = 0; kk < DL; ++kk) {
+                const int rk = sign_rank<DL>(g, kk) - (DL * G - d);
+                if (ok && rk >= 0 && rk < d) out[cell * d + rk] = S[kk];
+            }
+            return;
+        }
         sort_net<float, DL>(S);
         if constexpr (CTAB) {                 // mp_diag_ctab: last merge layer fused into the scan
             lane_merge<float, DL, G, true>(S, g);
