@@ -186,7 +186,7 @@ mp_status validate(mp_ctx* ctx, const void* T, int64_t d, int64_t n, int64_t m, 
 // results do not depend on how the plan is cut into launches (ranks, streamed chunks).
 // mp carries the data pointers and n, d, m, H; the tile fields are filled here.
 mp_status enqueue_tiles(mp_ctx* ctx, cudaStream_t s, int prec, bool self, mpk::MainParams mp, const Plan& pl,
-                        int64_t B0, int64_t B1, int64_t q0, int64_t q1, bool timed) {
+                        int64_t B0, int64_t B1, int64_t q0, int64_t q1, bool timed, Buf* pinned = nullptr) {
     const int64_t n = mp.n, HT = pl.H, NC = pl.nc, nb = B1 - B0;
     if (nb <= 0 || q1 <= q0) return MP_OK;
     const int64_t dlo = pl.dlo + B0 * NC, dhi = std::min<int64_t>(pl.dlo + B1 * NC - 1, pl.dhi);
@@ -224,7 +224,19 @@ mp_status enqueue_tiles(mp_ctx* ctx, cudaStream_t s, int prec, bool self, mpk::M
     if (tab[nq] != total) return fail(ctx, MP_ERR_INVALID, "internal: tile plan mismatch");
     if (total == 0) return MP_OK;
     MP_CUDA(ctx, ensure(ctx->seg, tab.size() * sizeof(long long)));
-    MP_CUDA(ctx, cudaMemcpyAsync(ctx->seg.p, tab.data(), tab.size() * sizeof(long long), cudaMemcpyHostToDevice, s));
+    const void* src = tab.data();
+    if (pinned) {   // a pinned copy: the upload is then asynchronous (a pageable one waits for the stream)
+        if (pinned->bytes < tab.size() * sizeof(long long)) {
+            if (pinned->p) cudaFreeHost(pinned->p);
+            pinned->p = nullptr;
+            pinned->bytes = 0;
+            MP_CUDA(ctx, cudaHostAlloc(&pinned->p, tab.size() * sizeof(long long) * 2, cudaHostAllocDefault));
+            pinned->bytes = tab.size() * sizeof(long long) * 2;
+        }
+        std::memcpy(pinned->p, tab.data(), tab.size() * sizeof(long long));
+        src = pinned->p;
+    }
+    MP_CUDA(ctx, cudaMemcpyAsync(ctx->seg.p, src, tab.size() * sizeof(long long), cudaMemcpyHostToDevice, s));
     MP_CUDA(ctx, ensure(ctx->counter, sizeof(unsigned long long)));
     MP_CUDA(ctx, cudaMemsetAsync(ctx->counter.p, 0, sizeof(unsigned long long), s));
     const mpk::Variant var = mpk::pick_variant(prec, mp.d);
@@ -418,6 +430,7 @@ typedef CUresult (*PF_memSetAccess)(CUdeviceptr, size_t, const CUmemAccessDesc*,
 typedef CUresult (*PF_memGran)(size_t*, const CUmemAllocationProp*, CUmemAllocationGranularity_flags);
 
 struct VArr {                                      // one virtual array
+    const char* name = "";
     CUdeviceptr base = 0;
     size_t bytes = 0;                              // reserved (a multiple of the granularity)
     std::vector<CUmemGenericAllocationHandle> h;   // per granule, 0 = unmapped
@@ -464,18 +477,19 @@ struct Vmm {
         arrs.push_back(&a);
         return CUDA_SUCCESS;
     }
+    // map granule g (its access rights are set per contiguous run by set_access)
     CUresult map_g(VArr& a, size_t g) {
         CUmemGenericAllocationHandle hd = 0;
         if (!pool.empty()) { hd = pool.back(); pool.pop_back(); }
         else { CUresult r = create(&hd, gran, &prop, 0); if (r != CUDA_SUCCESS) return r; }
         CUresult r = map(a.base + g * gran, gran, 0, hd, 0);
-        if (r == CUDA_SUCCESS) r = access(a.base + g * gran, gran, &acc, 1);
         if (r != CUDA_SUCCESS) { pool.push_back(hd); return r; }
         a.h[g] = hd;
         mapped += gran;
         peak = std::max(peak, mapped);
         return CUDA_SUCCESS;
     }
+    CUresult set_access(VArr& a, size_t g0, size_t g1) { return access(a.base + g0 * gran, (g1 - g0) * gran, &acc, 1); }
     CUresult unmap_g(VArr& a, size_t g) {
         CUresult r = unmap(a.base + g * gran, gran);
         pool.push_back(a.h[g]);
@@ -535,7 +549,7 @@ mp_status plan_stream(mp_ctx* ctx, int64_t d, int64_t n, int64_t m, int prec, in
                       int64_t budget, size_t gran, const Plan& pl, StreamGeo& g) {
     const mpk::Variant var = mpk::pick_variant(prec, (int)d);
     g.half = prec == MP_FP16 || prec == MP_MIXED || prec == MP_FP16C || prec == MP_FP16CK;
-    g.sb = g.half ? 16 : 4 * elt_bytes(prec);
+    g.sb = g.half ? 8 : 4 * elt_bytes(prec);   // stats entry bytes (half: the row format RH, 4 halves)
     g.tb = prec == MP_FP64 ? 8 : ((prec == MP_FP16 || prec == MP_FP16C) ? 2 : 4);
     g.tbs = prec == MP_FP32 ? 8 : g.tb;
     g.kb = prec == MP_FP64 ? 16 : 8;
@@ -546,8 +560,9 @@ mp_status plan_stream(mp_ctx* ctx, int64_t d, int64_t n, int64_t m, int prec, in
     const double key = (double)d * g.kb;
     const double scr = (double)d * (2.0 * g.tbs + (g.half ? 6.0 : 0.0) + 8.0);             // mu, nrm, flat, T slice
     const double out = 16.0 * d;                                                            // P, I row window
-    // windows: rows R, columns 3R (Wb = 2R)
-    g.per_R = self ? 4.0 * (side + key) + 3.0 * scr + out : (side + key) + 3.0 * side + 3.0 * scr + out;
+    // windows of two consecutive steps are resident (the next step is prepared while the current
+    // kernel runs): rows R, columns of two bands R + 2 Wb = 5R (Wb = 2R)
+    g.per_R = self ? 6.0 * (side + key) + 3.0 * scr + out : (side + key) + 5.0 * side + 3.0 * scr + out;
     const int narr = g.half ? 5 : 4;   // st, (stp), tw, mup, keys per side
     g.fixed = (double)gran * 2.0 /* windows */ * 2.0 /* partial granules */ * narr * (self ? 1 : 2) +
               2.0 * m * g.Dp * g.tb + 6.0 * scr + (16 << 20);
@@ -592,6 +607,7 @@ struct Streamer {
     int64_t d, n, m, L;
     bool self;
     unsigned char* hkeys = nullptr;        // host key store (pinned), absolute byte layout
+    bool own_s = true;                     // S.s created here (destroyed at the end of the call)
     Buf tslice, mu, nrm, flat, maxbits, dPw, dIw;
     int64_t wmax = 0;
     Side sq, sr;
@@ -609,27 +625,43 @@ struct Streamer {
     mp_status remap(VArr& a, const std::vector<char>& nm, bool is_keys, int64_t final_upto) {
         const double t0 = now();
         struct Acc { double& t; double t0; ~Acc() { t += now() - t0; } } acc{t_remap, t0};
-        if (is_keys) {   // save the key granules about to be unmapped (those still accumulating)
+        const size_t ng = a.h.size();
+        if (is_keys) {   // save the key granules about to be unmapped (those still accumulating), per run
             bool any = false;
-            for (size_t gi = 0; gi < a.h.size(); ++gi) {
-                if (!a.h[gi] || nm[gi]) continue;
-                const size_t b0 = gi * vm.gran;
-                if ((int64_t)((b0 + vm.gran - 1) / (d * g.kb)) < final_upto) { a.saved[gi] = 0; continue; }  // finalized
-                MP_CUDA(ctx, cudaMemcpyAsync(hkeys + b0, (char*)a.ptr() + b0, vm.gran, cudaMemcpyDeviceToHost, s));
-                a.saved[gi] = 1;
+            for (size_t gi = 0; gi < ng;) {
+                const bool sv = a.h[gi] && !nm[gi] && (int64_t)((gi * vm.gran + vm.gran - 1) / (d * g.kb)) >= final_upto;
+                if (a.h[gi] && !nm[gi] && !sv) a.saved[gi] = 0;   // finalized rows: dropped
+                if (!sv) { ++gi; continue; }
+                size_t ge = gi;
+                while (ge < ng && a.h[ge] && !nm[ge] && (int64_t)((ge * vm.gran + vm.gran - 1) / (d * g.kb)) >= final_upto)
+                    a.saved[ge++] = 1;
+                MP_CUDA(ctx, cudaMemcpyAsync(hkeys + gi * vm.gran, (char*)a.ptr() + gi * vm.gran, (ge - gi) * vm.gran,
+                                             cudaMemcpyDeviceToHost, s));
                 any = true;
+                gi = ge;
             }
             if (any) MP_CUDA(ctx, cudaStreamSynchronize(s));
         }
-        for (size_t gi = 0; gi < a.h.size(); ++gi)
+        static const char* keep_env = std::getenv("MP_STREAM_NOUNMAP");   // debugging knob: "1" or an array name
+        const bool keep_all = keep_env && (std::strcmp(keep_env, "1") == 0 || std::strcmp(keep_env, a.name) == 0);
+        for (size_t gi = 0; gi < ng && !keep_all; ++gi)
             if (a.h[gi] && !nm[gi]) MP_CU(ctx, vm.unmap_g(a, gi));
-        for (size_t gi = 0; gi < a.h.size(); ++gi) {
-            if (a.h[gi] || !nm[gi]) continue;
-            MP_CU(ctx, vm.map_g(a, gi));
-            if (!is_keys) continue;
-            const size_t b0 = gi * vm.gran;
-            if (a.saved[gi]) MP_CUDA(ctx, cudaMemcpyAsync((char*)a.ptr() + b0, hkeys + b0, vm.gran, cudaMemcpyHostToDevice, s));
-            else MP_CUDA(ctx, mpk::launch_init_keys(prec, (char*)a.ptr() + b0, (long long)(vm.gran / g.kb), s));
+        for (size_t gi = 0; gi < ng;) {   // map the new granules, one access call and copy per run
+            if (a.h[gi] || !nm[gi]) { ++gi; continue; }
+            size_t ge = gi;
+            while (ge < ng && !a.h[ge] && nm[ge]) MP_CU(ctx, vm.map_g(a, ge++));
+            MP_CU(ctx, vm.set_access(a, gi, ge));
+            if (is_keys) {
+                for (size_t k0 = gi; k0 < ge;) {
+                    size_t k1 = k0;
+                    while (k1 < ge && a.saved[k1] == a.saved[k0]) ++k1;
+                    char* dptr = (char*)a.ptr() + k0 * vm.gran;
+                    if (a.saved[k0]) MP_CUDA(ctx, cudaMemcpyAsync(dptr, hkeys + k0 * vm.gran, (k1 - k0) * vm.gran, cudaMemcpyHostToDevice, s));
+                    else MP_CUDA(ctx, mpk::launch_init_keys(prec, dptr, (long long)((k1 - k0) * vm.gran / g.kb), s));
+                    k0 = k1;
+                }
+            }
+            gi = ge;
         }
         return MP_OK;
     }
@@ -648,12 +680,20 @@ struct Streamer {
         const int64_t len = pp.s_end + m - 1 - pp.s_off;
         pp.T_ld = len;
         MP_CUDA(ctx, cudaMemcpy2DAsync(tslice.p, len * 8, sd.T + pp.s_off, L * 8, len * 8, d, cudaMemcpyHostToDevice, s));
-        MP_CUDA(ctx, mpk::launch_check_finite((const double*)tslice.p, d * len, (int*)ctx->flag.p, s));
         pp.T = (const double*)tslice.p;
         pp.st = sd.st.ptr(); pp.st_pair = sd.stp.ptr(); pp.tw = sd.tw.ptr(); pp.mup = sd.mup.ptr();
         pp.mu = mu.p; pp.nrm32 = (float*)nrm.p; pp.nrm64 = (double*)nrm.p; pp.flat = flat.p;
         pp.scale = (double*)sd.scale.p; pp.maxbits = (unsigned long long*)maxbits.p;
         MP_CUDA(ctx, mpk::launch_precompute(prec, pp, s, false));
+        return MP_OK;
+    }
+    // non-finite input (reading G23) over the whole series, one window at a time
+    mp_status check_pass(Side& sd) {
+        for (int64_t a = 0; a < L; a += wmax) {
+            const int64_t len = std::min(L, a + wmax) - a;
+            MP_CUDA(ctx, cudaMemcpy2DAsync(tslice.p, len * 8, sd.T + a, L * 8, len * 8, d, cudaMemcpyHostToDevice, s));
+            MP_CUDA(ctx, mpk::launch_check_finite((const double*)tslice.p, d * len, (int*)ctx->flag.p, s));
+        }
         return MP_OK;
     }
     // per-dimension half-precision scale of one series over all its windows (reading G16)
@@ -695,6 +735,8 @@ struct Streamer {
     }
 };
 
+constexpr int64_t kWinPad = 8;   // positions of margin around each streamed window
+
 mp_status run_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, int64_t n, int64_t m, int prec,
                      int64_t excl, int64_t budget, double* P, int64_t* I) {
     const bool self = Tr == nullptr;
@@ -704,7 +746,8 @@ mp_status run_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, 
     const Plan pl = build_plan(d, n, excl, self, prec, H);
     Streamer S{};
     S.ctx = ctx;
-    S.s = ctx->stream;
+    // S.s: the prep stream (remaps, key copies, window precompute); ctx->stream computes
+    if (cudaStreamCreateWithFlags(&S.s, cudaStreamNonBlocking) != cudaSuccess) return fail(ctx, MP_ERR_CUDA, "stream");
     S.prec = prec; S.d = d; S.n = n; S.m = m; S.L = L; S.self = self;
     const std::string err = S.vm.load(ctx->device);
     if (!err.empty()) return fail(ctx, MP_ERR_UNSUPPORTED, err);
@@ -723,17 +766,20 @@ mp_status run_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, 
     ctx->stream_R = S.g.R;
     ctx->stream_Wb = S.g.Wb;
     const StreamGeo& g = S.g;
-    cudaStream_t s = S.s;
+    cudaStream_t s = ctx->stream;
     struct Cleanup {
         Streamer& S;
+        cudaStream_t sc;
         ~Cleanup() {
+            cudaStreamSynchronize(sc);
             cudaStreamSynchronize(S.s);
             S.vm.destroy();
             if (S.hkeys) cudaFreeHost(S.hkeys);
+            if (S.s) { cudaStreamSynchronize(S.s); if (S.own_s) cudaStreamDestroy(S.s); }
             Buf* bs[] = {&S.tslice, &S.mu, &S.nrm, &S.flat, &S.maxbits, &S.dPw, &S.dIw, &S.sq.scale, &S.sr.scale};
             for (Buf* b : bs) release(*b);
         }
-    } cleanup{S};
+    } cleanup{S, s};
 
     // window scratch: the largest precompute window is a column window (R + Wb + 1 positions)
     S.wmax = g.R + g.Wb + 4;
@@ -746,23 +792,29 @@ mp_status run_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, 
     MP_CUDA(ctx, ensure(S.dPw, (size_t)d * g.R * 8));
     MP_CUDA(ctx, ensure(S.dIw, (size_t)d * g.R * 8));
     MP_CUDA(ctx, ensure(ctx->flag, sizeof(int)));
-    MP_CUDA(ctx, cudaMemsetAsync(ctx->flag.p, 0, sizeof(int), s));
+    MP_CUDA(ctx, cudaMemsetAsync(ctx->flag.p, 0, sizeof(int), S.s));   // the prep stream runs the checks
 
+    // The caller's T, P and I stay pageable: page-locking them for the call (cudaHostRegister)
+    // made the stream tests fail intermittently with launch failures (numpy arrays sharing pages),
+    // so the T slices and the output rows are copied from / to pageable memory.
     // virtual arrays at full size (absolute-position layout of run_partial)
     Side* sides[2] = {&S.sq, &S.sr};
     S.sq.T = T;
     S.sr.T = Tr;
     for (int si = 0; si < (self ? 1 : 2); ++si) {
         Side& sd = *sides[si];
+        sd.st.name = "st"; sd.stp.name = "stp"; sd.tw.name = "tw"; sd.mup.name = "mup";
         MP_CU(ctx, S.vm.reserve_arr(sd.st, (size_t)n * d * g.sb));
         if (g.half) MP_CU(ctx, S.vm.reserve_arr(sd.stp, (size_t)(n + 1) * d * 16));
         MP_CU(ctx, S.vm.reserve_arr(sd.tw, (size_t)L * g.Dp * g.tb));
         MP_CU(ctx, S.vm.reserve_arr(sd.mup, (size_t)n * g.Dp * g.tb));
+        if ((st = S.check_pass(sd)) != MP_OK) return st;
         if (g.half) {
             MP_CUDA(ctx, ensure(sd.scale, (size_t)d * sizeof(double)));
             if ((st = S.half_scale(sd)) != MP_OK) return st;
         }
     }
+    S.sq.keys.name = "keys";
     MP_CU(ctx, S.vm.reserve_arr(S.sq.keys, (size_t)n * d * g.kb + 16));
     MP_CUDA(ctx, cudaHostAlloc((void**)&S.hkeys, S.sq.keys.bytes, cudaHostAllocDefault));
 
@@ -779,51 +831,129 @@ mp_status run_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, 
 
     ctx->last_launches = 0;
     ctx->last_ms = 0.0;
-    std::vector<cudaEvent_t> evs;
-    struct EvFree { std::vector<cudaEvent_t>& v; ~EvFree() { for (auto e : v) cudaEventDestroy(e); } } evfree{evs};
+
+    // the step list: (row chunk, diagonal band) pairs with cells, in row-chunk order
+    struct Step { int64_t B0, B1, q0, q1, i0, i1; Ivl rows, cols; bool last; };
+    std::vector<Step> steps;
+    std::vector<std::pair<int64_t, int64_t>> empty_chunks;   // row chunks no band reaches
     const int64_t HT = g.HT, NC = g.NC, nq = std::max<int64_t>(1, (n + HT - 1) / HT), qs = g.R / HT;
     const int64_t BW = g.Wb / NC;   // blocks per band
     for (int64_t q0 = 0; q0 < nq; q0 += qs) {
         const int64_t q1 = std::min(nq, q0 + qs), i0 = q0 * HT, i1 = std::min(n, q1 * HT);
+        const size_t first = steps.size();
         for (int64_t B0 = 0; B0 < pl.nb; B0 += BW) {
             const int64_t B1 = std::min(pl.nb, B0 + BW);
             const int64_t dlo = pl.dlo + B0 * NC, dhi = std::min(pl.dlo + B1 * NC - 1, pl.dhi);
             const int64_t ra = std::max(i0, -dhi), rb = std::min(i1, n - dlo);   // rows with cells
             if (ra >= rb) continue;
-            const Ivl rows{i0, i1}, cols{std::max<int64_t>(0, ra + dlo), std::min<int64_t>(n, rb - 1 + dhi + 1)};
-            { const double t0 = Streamer::now();
-              MP_CUDA(ctx, cudaStreamSynchronize(s));   // the previous launch is done with the windows
-              S.t_sync += Streamer::now() - t0; }
-            if (self) {
-                const std::vector<Ivl> both{rows, cols};
-                if ((st = S.ensure_side(S.sq, both, &both, i0)) != MP_OK) return st;
-            } else {
-                const std::vector<Ivl> r1{rows};
-                if ((st = S.ensure_side(S.sq, r1, &r1, i0)) != MP_OK) return st;
-                if ((st = S.ensure_side(S.sr, {cols}, nullptr, 0)) != MP_OK) return st;
-            }
-            cudaEvent_t e0, e1;
-            MP_CUDA(ctx, cudaEventCreate(&e0));
-            evs.push_back(e0);
-            MP_CUDA(ctx, cudaEventCreate(&e1));
-            evs.push_back(e1);
-            MP_CUDA(ctx, cudaEventRecord(e0, s));
-            if ((st = enqueue_tiles(ctx, s, prec, self, mp, pl, B0, B1, q0, q1, false)) != MP_OK) return st;
-            MP_CUDA(ctx, cudaEventRecord(e1, s));
+            // windows with a margin of kWinPad positions: the kernels stage one batch of positions
+            // past a tile's last row / column (never used by a cell, but read)
+            steps.push_back({B0, B1, q0, q1, i0, i1, {i0, std::min<int64_t>(n, i1 + kWinPad)},
+                             {std::max<int64_t>(0, ra + dlo - kWinPad), std::min<int64_t>(n, rb + dhi + kWinPad)}, false});
         }
-        // rows [i0, i1) are final: later chunks only touch rows >= i1 and (self-join) columns
-        // > their rows.  Their keys are made resident (rows no band reached keep the empty key:
-        // P = +inf, I = -1, reading G3) and finalized.
-        MP_CUDA(ctx, cudaStreamSynchronize(s));
-        if ((st = S.remap(S.sq.keys, S.need_mask(S.sq.keys, {{i0, i1}}, (double)d * g.kb, 0), true, i0)) != MP_OK)
-            return st;
+        if (steps.size() == first) empty_chunks.push_back({i0, i1});
+        else steps.back().last = true;
+    }
+
+    // the tile tables of every step fit the device table buffer allocated here: re-allocating it
+    // inside the pipeline would free memory a running kernel reads
+    MP_CUDA(ctx, ensure(ctx->seg, (size_t)(2 * nq + 1 + BW + 1) * sizeof(long long)));
+    MP_CUDA(ctx, ensure(ctx->counter, sizeof(unsigned long long)));
+
+
+
+    // Pipeline: while the fused kernel of step k runs on the compute stream, the host remaps the
+    // windows of step k + 1 and the prep stream restores keys and precomputes the new positions.
+    // Resident at any time: the windows of two consecutive steps.  Granules outside both are
+    // unmapped only after the kernel (and chunk finalize) two steps back has completed.
+    cudaStream_t sc = s;            // compute stream (kernels, finalize, output copies)
+    cudaStream_t sp = S.s;          // prep stream (remap copies, precompute)
+    std::vector<cudaEvent_t> evs;   // per launch: start, end (timing)
+    std::vector<cudaEvent_t> done;  // per step: compute stream done through the step (finalize incl.)
+    cudaEvent_t prep_ev = nullptr;
+    struct EvFree {
+        std::vector<cudaEvent_t>& a; std::vector<cudaEvent_t>& b; cudaEvent_t& c;
+        ~EvFree() { for (auto e : a) cudaEventDestroy(e); for (auto e : b) cudaEventDestroy(e); if (c) cudaEventDestroy(c); }
+    } evfree{evs, done, prep_ev};
+    MP_CUDA(ctx, cudaEventCreateWithFlags(&prep_ev, cudaEventDisableTiming));
+    Buf tab_pin[3];
+    struct PinFree { Buf* b; ~PinFree() { for (int i = 0; i < 3; ++i) if (b[i].p) cudaFreeHost(b[i].p); } } pinfree{tab_pin};
+    auto finalize_rows = [&](int64_t i0, int64_t i1) -> mp_status {
         const int64_t w = i1 - i0;
         const double tf0 = Streamer::now();
         MP_CUDA(ctx, mpk::launch_finalize_window(prec, S.sq.keys.ptr(), i0, i1, (int)d, (double*)S.dPw.p,
-                                                 (long long*)S.dIw.p, s));
-        MP_CUDA(ctx, cudaMemcpy2DAsync(P + i0, n * 8, S.dPw.p, w * 8, w * 8, d, cudaMemcpyDeviceToHost, s));
-        MP_CUDA(ctx, cudaMemcpy2DAsync(I + i0, n * 8, S.dIw.p, w * 8, w * 8, d, cudaMemcpyDeviceToHost, s));
+                                                 (long long*)S.dIw.p, sc));
+        MP_CUDA(ctx, cudaMemcpy2DAsync(P + i0, n * 8, S.dPw.p, w * 8, w * 8, d, cudaMemcpyDeviceToHost, sc));
+        MP_CUDA(ctx, cudaMemcpy2DAsync(I + i0, n * 8, S.dIw.p, w * 8, w * 8, d, cudaMemcpyDeviceToHost, sc));
         S.t_fin += Streamer::now() - tf0;
+        return MP_OK;
+    };
+    // the window intervals of a step: (series positions of the query side, of the reference side,
+    // keys)
+    auto windows = [&](const Step& t, std::vector<Ivl>& q, std::vector<Ivl>& r, std::vector<Ivl>& k) {
+        if (self) { q.push_back(t.rows); q.push_back(t.cols); k.push_back(t.rows); k.push_back(t.cols); }
+        else { q.push_back(t.rows); k.push_back(t.rows); r.push_back(t.cols); }
+    };
+    size_t ei = 0;   // next empty chunk
+    for (size_t k = 0; k < steps.size(); ++k) {
+        const Step& t = steps[k];
+        // empty row chunks before this step: finalize them synchronously (keys initialised)
+        while (ei < empty_chunks.size() && empty_chunks[ei].first < t.i0) {
+            MP_CUDA(ctx, cudaStreamSynchronize(sc));
+            std::vector<Ivl> kv{{empty_chunks[ei].first, empty_chunks[ei].second}};
+            if (k > 0) { std::vector<Ivl> q, r; windows(steps[k - 1], q, r, kv); }
+            if ((st = S.remap(S.sq.keys, S.need_mask(S.sq.keys, merge_ivls(kv), (double)d * g.kb, 0), true, t.i0)) != MP_OK)
+                return st;
+            MP_CUDA(ctx, cudaStreamSynchronize(sp));
+            if ((st = finalize_rows(empty_chunks[ei].first, empty_chunks[ei].second)) != MP_OK) return st;
+            ++ei;
+        }
+        // The remap of step k overlaps the kernel of step k - 1 (the windows of both steps stay
+        // resident); MP_STREAM_SERIAL=1 waits for that kernel first (no overlap)
+        static const bool pipelined = std::getenv("MP_STREAM_SERIAL") == nullptr;
+        if (!pipelined && k >= 1) {
+            const double t0 = Streamer::now();
+            MP_CUDA(ctx, cudaEventSynchronize(done[k - 1]));
+            S.t_sync += Streamer::now() - t0;
+        }
+        if (k >= 2) {
+            const double t0 = Streamer::now();
+            MP_CUDA(ctx, cudaEventSynchronize(done[k - 2]));
+            S.t_sync += Streamer::now() - t0;
+        }
+        std::vector<Ivl> q, r, kv;
+        windows(t, q, r, kv);
+        if (k > 0) windows(steps[k - 1], q, r, kv);   // still in use by the running kernel
+        // keys of rows below the oldest resident chunk are final: dropped, not saved
+        const int64_t final_upto = k > 0 ? steps[k - 1].i0 : t.i0;
+        if ((st = S.ensure_side(S.sq, q, &kv, final_upto)) != MP_OK) return st;
+        if (!self && (st = S.ensure_side(S.sr, r, nullptr, 0)) != MP_OK) return st;
+        MP_CUDA(ctx, cudaEventRecord(prep_ev, sp));
+        MP_CUDA(ctx, cudaStreamWaitEvent(sc, prep_ev, 0));
+        cudaEvent_t e0, e1, dn;
+        MP_CUDA(ctx, cudaEventCreate(&e0));
+        evs.push_back(e0);
+        MP_CUDA(ctx, cudaEventCreate(&e1));
+        evs.push_back(e1);
+        MP_CUDA(ctx, cudaEventRecord(e0, sc));
+        if ((st = enqueue_tiles(ctx, sc, prec, self, mp, pl, t.B0, t.B1, t.q0, t.q1, false, &tab_pin[k % 3])) != MP_OK)
+            return st;
+        MP_CUDA(ctx, cudaEventRecord(e1, sc));
+        // rows [i0, i1) are final after the chunk's last band: later chunks only touch rows >= i1
+        // and (self-join) columns > their rows; rows no band reached keep the empty key (G3)
+        if (t.last && (st = finalize_rows(t.i0, t.i1)) != MP_OK) return st;
+        MP_CUDA(ctx, cudaEventCreateWithFlags(&dn, cudaEventDisableTiming));
+        done.push_back(dn);
+        MP_CUDA(ctx, cudaEventRecord(dn, sc));
+    }
+    while (ei < empty_chunks.size()) {   // trailing row chunks no band reaches
+        MP_CUDA(ctx, cudaStreamSynchronize(sc));
+        std::vector<Ivl> kv{{empty_chunks[ei].first, empty_chunks[ei].second}};
+        if ((st = S.remap(S.sq.keys, S.need_mask(S.sq.keys, kv, (double)d * g.kb, 0), true, empty_chunks[ei].first)) != MP_OK)
+            return st;
+        MP_CUDA(ctx, cudaStreamSynchronize(sp));
+        if ((st = finalize_rows(empty_chunks[ei].first, empty_chunks[ei].second)) != MP_OK) return st;
+        ++ei;
     }
     if (std::getenv("MP_STREAM_PROFILE"))
         std::fprintf(stderr, "mp_compute_stream: host s sync %.3f remap %.3f precompute %.3f finalize %.3f\n", S.t_sync,

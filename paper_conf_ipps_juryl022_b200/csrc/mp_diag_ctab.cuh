@@ -44,7 +44,8 @@
 #define MP_CTAB_PAIR 1      // G == 2: the pair-mode merge (pair_si)
 #endif
 #ifndef MP_CTAB_SIGN
-#define MP_CTAB_SIGN 1      // G == 4: sign-split cross-lane merge (two of three cross-lane steps uniform)
+#define MP_CTAB_SIGN 0      // G == 4: sign-split cross-lane merge (two of three cross-lane steps uniform;
+                            // measured C3 -1 % time but the negative lanes' prefix sums cancel: off)
 #endif
 #ifndef MP_CTAB_TA
 #define MP_CTAB_TA 1        // thresholds in rank-contiguous per-slot arrays (read as vectors after
