@@ -8,5 +8,5 @@ python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.txt 2>&1; 
 timeout 1800 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err; tail -2 gpurun_out/bench_default.err; cut -c1-300 gpurun_out/bench_default.json
 timeout 900 python bench.py --impl reference > gpurun_out/bench_reference.json 2> gpurun_out/bench_reference.err; cut -c1-200 gpurun_out/bench_reference.json
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-per-precision --no-per-config --no-context --no-stream > gpurun_out/bench_under_ncu.txt 2>&1; tail -1 gpurun_out/bench_under_ncu.txt | cut -c1-200
-MP_SEED_MODE=tc timeout 900 ncu --set full --clock-control none --import-source on -k regex:seed_gemm -s 1 -c 1 -o gpurun_out/full_X64_seed_gemm python scripts/prof_one.py X64_32768_256 mixed 1 > gpurun_out/ncu_seed_gemm.log 2>&1; tail -1 gpurun_out/ncu_seed_gemm.log
+echo skip-ncu
 exit 0
