@@ -1,0 +1,9 @@
+// Explicit instantiations of the fused diagonal kernel (split across translation units
+// so the template variants compile in parallel; see build.py).
+#define MP_DIAG_IMPL
+#include "mp_diag.cuh"
+namespace mpk {
+template struct Inst<float, 1, 1, 2, false, false>;
+template struct Inst<float, 2, 1, 2, false, false>;
+template struct Inst<float, 4, 1, 2, false, false>;
+}  // namespace mpk

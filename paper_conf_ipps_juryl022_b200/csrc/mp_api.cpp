@@ -264,6 +264,14 @@ mp_status enqueue_tiles(mp_ctx* ctx, cudaStream_t s, int prec, bool self, mpk::M
     return MP_OK;
 }
 
+// FP32 windows shorter than kCompMinM run the plain QT recurrence in the warp kernels (P32N): the
+// compensated one (reading R4) is needed for the 1e-4 gate at m >= 256 only
+// (C2 FP32: 45.4 -> 44.4 ms without it).  The block kernels (d >= 64) always compensate.
+constexpr int64_t kCompMinM = 192;
+int kernel_prec(int prec, int64_t m, const mpk::Variant& var) {
+    return (prec == MP_FP32 && m < kCompMinM && !var.cta && !var.ctab) ? (int)mpk::P32N : prec;
+}
+
 // Tensor-core seeds apply to the FP32-precalc half modes (Mixed, FP16CK) on the block kernels.
 // seed table per row chunk (device bytes): up to 128 seed rows (one MMA tile of M = 128) per chunk,
 // so each Hankel operand tile the GEMM builds serves as many rows as fit
@@ -361,7 +369,7 @@ mp_status run_partial(mp_ctx* ctx, cudaStream_t s, const double* dT, const doubl
         mp.n = n; mp.d = (int)d; mp.m = (int)m; mp.H = (int)H;
         const int64_t nq = std::max<int64_t>(1, (n + pl.H - 1) / pl.H);
         if (!(tc_seeds(ctx, prec) && var.cta))
-            return enqueue_tiles(ctx, s, prec, self, mp, pl, bb[rank], bb[rank + 1], 0, nq, true);
+            return enqueue_tiles(ctx, s, kernel_prec(prec, m, var), self, mp, pl, bb[rank], bb[rank + 1], 0, nq, true);
         // tensor-core seeds (NEXT-3): per row chunk, one seed GEMM for the chunk's re-seed rows,
         // then the fused kernel over the chunk's tiles reading the table
         const int64_t B0 = bb[rank], B1 = bb[rank + 1];
@@ -936,7 +944,8 @@ mp_status run_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, 
         MP_CUDA(ctx, cudaEventCreate(&e1));
         evs.push_back(e1);
         MP_CUDA(ctx, cudaEventRecord(e0, sc));
-        if ((st = enqueue_tiles(ctx, sc, prec, self, mp, pl, t.B0, t.B1, t.q0, t.q1, false, &tab_pin[k % 3])) != MP_OK)
+        if ((st = enqueue_tiles(ctx, sc, kernel_prec(prec, m, mpk::pick_variant(prec, (int)d)), self, mp, pl, t.B0, t.B1,
+                                t.q0, t.q1, false, &tab_pin[k % 3])) != MP_OK)
             return st;
         MP_CUDA(ctx, cudaEventRecord(e1, sc));
         // rows [i0, i1) are final after the chunk's last band: later chunks only touch rows >= i1

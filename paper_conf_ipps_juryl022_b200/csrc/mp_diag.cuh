@@ -438,7 +438,9 @@ template <class T, int DL, int G, int W> constexpr int min_blocks() {
     // caps the register budget where ptxas still fits without spills (measured with -Xptxas -v)
     return (sizeof(T) == 4 && G == 1 && DL * W <= 16) ? MP_MINB_F32 : MP_MINB;
 }
-template <class T, int DL, int G, int W, bool SELF>
+// COMP: the compensated QT recurrence (reading R4); off for short windows (m < kCompMinM in
+// mp_api.cpp), where the plain FP32 recurrence is inside the 1e-4 gate
+template <class T, int DL, int G, int W, bool SELF, bool COMP = true>
 __global__ void __launch_bounds__(128, (min_blocks<T, DL, G, W>()))
 mp_diag(const MainParams p) {
     using V4 = typename PT<T>::V4;
@@ -642,8 +644,8 @@ mp_diag(const MainParams p) {
 #pragma unroll
                 for (int kk = 0; kk < SC; ++kk) {  // the Kahan sum is acc - cmp: keep both words
                     const bool pad = ((c0 + kk) * G + g) >= d;  // padded dims: zero data
-                    QT[u][c0 + kk] = pad ? (T)-1 : acc[kk];
-                    QL[u][c0 + kk] = pad ? (T)0 : -cmp[kk];
+                    QT[u][c0 + kk] = pad ? (T)-1 : (COMP ? acc[kk] : acc[kk] - cmp[kk]);
+                    QL[u][c0 + kk] = pad ? (T)0 : (COMP ? -cmp[kk] : (T)0);
                 }
             }
         };
@@ -709,15 +711,25 @@ mp_diag(const MainParams p) {
                 const V4 C = colv[pl * PSC + scn];
                 if constexpr (W == 2) {
                     const V4 C0v = Cold[kk];
-                    if (upd[0]) QL[0][kk] = fma(R.x, C0v.y, fma(C0v.x, R.y, QL[0][kk]));   // Eq. (1)
                     const T pr0 = R.z * C0v.z;
-                    S[0][kk] = PT<T>::sqrt_abs(fma(-QL[0][kk], pr0, fma(-QT[0][kk], pr0, two_m)));
+                    if constexpr (COMP) {
+                        if (upd[0]) QL[0][kk] = fma(R.x, C0v.y, fma(C0v.x, R.y, QL[0][kk]));   // Eq. (1)
+                        S[0][kk] = PT<T>::sqrt_abs(fma(-QL[0][kk], pr0, fma(-QT[0][kk], pr0, two_m)));
+                    } else {
+                        if (upd[0]) QT[0][kk] = fma(R.x, C0v.y, fma(C0v.x, R.y, QT[0][kk]));   // Eq. (1)
+                        S[0][kk] = PT<T>::sqrt_abs(fma(-QT[0][kk], pr0, two_m));
+                    }
                     if constexpr (KEEP) tc0[kk] = C0v.w;
                     Cnew[kk] = C;
                 }
-                if (upd[W - 1]) QL[W - 1][kk] = fma(R.x, C.y, fma(C.x, R.y, QL[W - 1][kk]));  // Eq. (1)
                 const T pr = R.z * C.z;
-                S[W - 1][kk] = PT<T>::sqrt_abs(fma(-QL[W - 1][kk], pr, fma(-QT[W - 1][kk], pr, two_m)));  // Eq. (1)
+                if constexpr (COMP) {
+                    if (upd[W - 1]) QL[W - 1][kk] = fma(R.x, C.y, fma(C.x, R.y, QL[W - 1][kk]));  // Eq. (1)
+                    S[W - 1][kk] = PT<T>::sqrt_abs(fma(-QL[W - 1][kk], pr, fma(-QT[W - 1][kk], pr, two_m)));  // Eq. (1)
+                } else {
+                    if (upd[W - 1]) QT[W - 1][kk] = fma(R.x, C.y, fma(C.x, R.y, QT[W - 1][kk]));  // Eq. (1)
+                    S[W - 1][kk] = PT<T>::sqrt_abs(fma(-QT[W - 1][kk], pr, two_m));                // Eq. (1)
+                }
                 if constexpr (KEEP) {
                     tr[kk] = R.w;
                     if constexpr (W == 1) tc0[kk] = C.w;
@@ -914,7 +926,7 @@ mp_diag(const MainParams p) {
 
         int to_seed = H;  // steps until the next re-seed (H is a multiple of SB)
         for (int s0 = 0; s0 < s_end; s0 += SB) {
-            if ((s0 & (FOLD - 1)) == 0) {  // fold the increments into QT (exact Fast2Sum)
+            if (COMP && (s0 & (FOLD - 1)) == 0) {  // fold the increments into QT (exact Fast2Sum)
 #pragma unroll
                 for (int u = 0; u < W; ++u)
 #pragma unroll
@@ -969,7 +981,7 @@ mp_diag(const MainParams p) {
     }
 }
 
-template <class T, int DL, int G, int W, bool SELF> struct Inst {
+template <class T, int DL, int G, int W, bool SELF, bool COMP = true> struct Inst {
     static size_t smem();
     static cudaError_t launch(const MainParams& p, int grid, cudaStream_t s);
     static int blocks_per_sm();
@@ -977,22 +989,22 @@ template <class T, int DL, int G, int W, bool SELF> struct Inst {
 };
 
 #ifdef MP_DIAG_IMPL
-template <class T, int DL, int G, int W, bool SELF> size_t Inst<T, DL, G, W, SELF>::smem() {
+template <class T, int DL, int G, int W, bool SELF, bool COMP> size_t Inst<T, DL, G, W, SELF, COMP>::smem() {
     return Smem<T, DL, G, W>::bytes_per_warp * Smem<T, DL, G, W>::WPB;
 }
-template <class T, int DL, int G, int W, bool SELF>
-cudaError_t Inst<T, DL, G, W, SELF>::launch(const MainParams& p, int grid, cudaStream_t s) {
+template <class T, int DL, int G, int W, bool SELF, bool COMP>
+cudaError_t Inst<T, DL, G, W, SELF, COMP>::launch(const MainParams& p, int grid, cudaStream_t s) {
     const size_t sm = smem();
-    cudaError_t e = cudaFuncSetAttribute(mp_diag<T, DL, G, W, SELF>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaError_t e = cudaFuncSetAttribute(mp_diag<T, DL, G, W, SELF, COMP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
-    mp_diag<T, DL, G, W, SELF><<<grid, Smem<T, DL, G, W>::WPB * 32, sm, s>>>(p);
+    mp_diag<T, DL, G, W, SELF, COMP><<<grid, Smem<T, DL, G, W>::WPB * 32, sm, s>>>(p);
     return cudaGetLastError();
 }
-template <class T, int DL, int G, int W, bool SELF> int Inst<T, DL, G, W, SELF>::blocks_per_sm() {
+template <class T, int DL, int G, int W, bool SELF, bool COMP> int Inst<T, DL, G, W, SELF, COMP>::blocks_per_sm() {
     const size_t sm = smem();
-    cudaFuncSetAttribute(mp_diag<T, DL, G, W, SELF>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaFuncSetAttribute(mp_diag<T, DL, G, W, SELF, COMP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     int nb = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mp_diag<T, DL, G, W, SELF>, Smem<T, DL, G, W>::WPB * 32, sm);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mp_diag<T, DL, G, W, SELF, COMP>, Smem<T, DL, G, W>::WPB * 32, sm);
     return nb;
 }
 #endif

@@ -84,7 +84,8 @@ struct PreParams {
 };
 
 // Precision codes match mp_precision.
-enum { P64 = 0, P32 = 1, P16 = 2, PMIX = 3, P16C = 4, P16CK = 5 };
+// P32N (kernel-internal): FP32 with the plain QT recurrence, chosen for short windows (warp kernels)
+enum { P64 = 0, P32 = 1, P16 = 2, PMIX = 3, P16C = 4, P16CK = 5, P32N = 6 };
 
 // Variant selection for a given (precision, d): dims per lane DL and lanes per cell G.
 struct Variant { int DL; int G; int W; int NC; int cta = 0; /* warps per block of the block-cooperative kernel, 0: warp tiles */

@@ -366,6 +366,7 @@ Variant pick_variant(int prec, int d) {
     // A lane holds DL <= 16 dims (register budget; DL = 32 only for FP32 d > 512); for small
     // d a lane owns W = 2 adjacent diagonals (d <= 8).
     if (prec == P16CK) prec = PMIX;   // same kernels as Mixed
+    if (prec == P32N) prec = P32;     // same shapes as FP32
     int dp = 1;
     while (dp < d) dp <<= 1;
     Variant v;
@@ -396,14 +397,14 @@ Variant pick_variant(int prec, int d) {
 }
 
 // op: 0 = smem, 1 = launch, 2 = blocks/SM, 3 = warps/block
-template <class T, bool SELF>
+template <class T, bool SELF, bool COMP = true>
 static long long dispatch_t(int op, int DL, int G, int W, const MainParams* p, int grid, cudaStream_t s) {
 #define MP_CASE(dl, g, w)                                                                  \
     if (DL == dl && G == g && W == w) {                                                    \
-        if (op == 0) return (long long)Inst<T, dl, g, w, SELF>::smem();                    \
-        if (op == 1) return (long long)Inst<T, dl, g, w, SELF>::launch(*p, grid, s);       \
-        if (op == 3) return Inst<T, dl, g, w, SELF>::warps_per_block();                    \
-        return Inst<T, dl, g, w, SELF>::blocks_per_sm();                                   \
+        if (op == 0) return (long long)Inst<T, dl, g, w, SELF, COMP>::smem();              \
+        if (op == 1) return (long long)Inst<T, dl, g, w, SELF, COMP>::launch(*p, grid, s); \
+        if (op == 3) return Inst<T, dl, g, w, SELF, COMP>::warps_per_block();              \
+        return Inst<T, dl, g, w, SELF, COMP>::blocks_per_sm();                             \
     }
     if constexpr (sizeof(T) == 4) {
         MP_CASE(1, 1, 2) MP_CASE(2, 1, 2) MP_CASE(4, 1, 2) MP_CASE(8, 1, 2) MP_CASE(16, 1, 1)
@@ -536,6 +537,7 @@ static long long dispatch(int op, int prec, bool self, int d, const MainParams* 
     if (prec == P16CK) return self ? dispatch_h<true, 3>(op, v.DL, v.G, p, grid, s) : dispatch_h<false, 3>(op, v.DL, v.G, p, grid, s);
     if (prec == P64) return self ? dispatch_64f<true>(op, v.DL, v.G, p, grid, s) : dispatch_64f<false>(op, v.DL, v.G, p, grid, s);
     if (prec == P32) return self ? dispatch_t<float, true>(op, v.DL, v.G, v.W, p, grid, s) : dispatch_t<float, false>(op, v.DL, v.G, v.W, p, grid, s);
+    if (prec == P32N) return self ? dispatch_t<float, true, false>(op, v.DL, v.G, v.W, p, grid, s) : dispatch_t<float, false, false>(op, v.DL, v.G, v.W, p, grid, s);
     return op == 1 ? (long long)cudaErrorInvalidValue : 0;
 }
 
