@@ -61,8 +61,13 @@ template <int DL, int G, int NW> struct CtaGeoH {
     static constexpr size_t col_bytes = (size_t)RC * D * sizeof(H4);
     static constexpr size_t row_bytes = a16((size_t)RR * D * sizeof(RH));
     static constexpr size_t stg_bytes = a16((size_t)(RR + RC) * D * sizeof(float));
-    static constexpr size_t bytes = col_bytes + row_bytes + stg_bytes + 16;
+    static constexpr size_t bytes = col_bytes + row_bytes + stg_bytes + 16 /* tile index */ + 16 /* mbarrier */;
 };
+
+#ifndef MP_CTAH_TMA
+#define MP_CTAH_TMA 0   // stage each entering position's statistics by one TMA bulk copy (measured:
+                        // C3 Mixed 3529 -> 3701 ms, X64 60.1 -> 62.8 ms against cp.async: off)
+#endif
 
 // Seeds of a cell pair from the tensor-core seed table (MP_SEEDS_TC, mp_seed_tc.cu) when every
 // valid cell of the pair starts on a table row (a re-seed row r H inside the table's row range
@@ -109,6 +114,7 @@ mp_diag_cta_h(const MainParams p) {
     float* rowb = reinterpret_cast<float*>(smem_raw + Cg::col_bytes + Cg::row_bytes);
     float* colb = rowb + (size_t)RR * D;
     long long* tile_sh = reinterpret_cast<long long*>(smem_raw + Cg::col_bytes + Cg::row_bytes + Cg::stg_bytes);
+    unsigned long long* bar = reinterpret_cast<unsigned long long*>(smem_raw + Cg::col_bytes + Cg::row_bytes + Cg::stg_bytes + 16);
 
     const RH* __restrict__ st_q = reinterpret_cast<const RH*>(p.st_q);   // row format [pos][dim]
     const H4* __restrict__ st_r = reinterpret_cast<const H4*>(p.st_r);   // pair format [pos + 1][dim]
@@ -133,8 +139,51 @@ mp_diag_cta_h(const MainParams p) {
     auto rslot = [&](int pos) { return (pos + off_r) % RR; };
     auto cslot = [&](int pos) { return (pos + off_c) % RC; };
 
-    // stage positions [p_lo, p_hi) (relative to base) of one side: stats by cp.async, the
-    // threshold (value word of the merge key) into the float staging slot
+    // TMA staging (MP_CTAH_TMA, d even so a position's d row entries of 8 B are whole 16-byte
+    // units): one cp.async.bulk per entering position and side, issued by thread 0, completing
+    // on the block's mbarrier (armed once per batch with the batch's byte count).  The padded
+    // planes [d, D) of every slot never change and are written once; the thresholds still come
+    // from the merge keys by cp.async and are converted after the batch (fixup).
+    const bool tma = MP_CTAH_TMA && (d % 2) == 0;
+    unsigned phase = 0;
+    if (tma) {
+        for (int e = tid; e < (RR + RC) * (D - d); e += NT) {
+            const int sl = e / (D - d), pl = d + e % (D - d);
+            if (sl < RR) {
+                RH* dst = &rowv[sl * D + pl];
+                dst->df = HZERO; dst->dg = HZERO; dst->a = HINF;
+            } else {
+                H4* dst = &colv[(sl - RR) * D + pl];
+                dst->x = __half2half2(HZERO); dst->y = dst->x; dst->z = __half2half2(HINF);
+            }
+        }
+        if (tid == 0) {
+            mbar_init(bar, 1);
+            fence_proxy_async();
+        }
+    }
+    auto tma_issue = [&](int R0_, int r_lo, int r_hi, int C0_, int c_lo, int c_hi) {
+        if (tid != 0) return;
+        const unsigned rb = (unsigned)d * 8u, cb = (unsigned)d * 16u;
+        unsigned bytes = 0;
+        for (int q = r_lo; q < r_hi; ++q) bytes += rb;   // rows are always in range
+        for (int q = c_lo; q < c_hi; ++q) {
+            const int pos = C0_ + q;
+            if (pos >= -1 && pos < n32) bytes += cb;
+        }
+        mbar_arrive_expect_tx(bar, bytes);
+        for (int q = r_lo; q < r_hi; ++q) {
+            const int pos = R0_ + q;
+            bulk_g2s(&rowv[rslot(pos) * D], st_q + (size_t)pos * d, rb, bar);
+        }
+        for (int q = c_lo; q < c_hi; ++q) {
+            const int pos = C0_ + q;
+            if (pos >= -1 && pos < n32) bulk_g2s(&colv[cslot(pos) * D], st_r + (size_t)(pos + 1) * d, cb, bar);
+        }
+    };
+
+    // stage positions [p_lo, p_hi) (relative to base) of one side: stats by cp.async (unless
+    // TMA stages them), the threshold (value word of the merge key) into the float staging slot
     auto stage = [&](bool is_row, int base, int p_lo, int p_hi) {
         const int cnt = p_hi - p_lo;
         for (int e = tid; e < cnt * D; e += NT) {
@@ -144,7 +193,9 @@ mp_diag_cta_h(const MainParams p) {
             if (is_row) {
                 const int ix = rslot(pos) * D + pl;
                 RH* dst = &rowv[ix];
-                if (pos >= 0 && pos < n32 && pl < d) {
+                if (tma) {
+                    // statistics by TMA (padded planes preset)
+                } else if (pos >= 0 && pos < n32 && pl < d) {
                     cp_async8(dst, st_q + (size_t)pos * d + pl);      // (df, dg, a, -)
                 } else {  // padded dimension / past the end: a = +inf with QT = -1 gives D = +inf
                     dst->df = HZERO; dst->dg = HZERO; dst->a = HINF;
@@ -156,11 +207,14 @@ mp_diag_cta_h(const MainParams p) {
             } else {
                 const int ix = cslot(pos) * D + pl;
                 H4* dst = &colv[ix];
-                if (pos >= -1 && pos < n32 && pl < d) {
-                    const H4* src = st_r + (size_t)(pos + 1) * d + pl;  // pair (pos, pos + 1)
-                    cp_async8(dst, src);
-                    cp_async4(&dst->z, &src->z);
-                } else {
+                const bool in = pos >= -1 && pos < n32;
+                if (in && pl < d) {
+                    if (!tma) {
+                        const H4* src = st_r + (size_t)(pos + 1) * d + pl;  // pair (pos, pos + 1)
+                        cp_async8(dst, src);
+                        cp_async4(&dst->z, &src->z);
+                    }
+                } else if (!(tma && in)) {   // TMA: padded planes of in-range positions are preset
                     dst->x = __half2half2(HZERO); dst->y = dst->x; dst->z = __half2half2(HINF);
                 }
                 if (SELF && pos >= 0 && pos < n32 && rk < d)
@@ -190,6 +244,7 @@ mp_diag_cta_h(const MainParams p) {
     };
 
     for (;;) {
+        if (tma) fence_proxy_async();   // this thread's generic ring writes precede later bulk copies
         __syncthreads();  // previous tile fully done (rings, tile_sh)
         if (tid == 0) *tile_sh = (long long)atomicAdd(p.counter, 1ull);
         __syncthreads();
@@ -233,10 +288,12 @@ mp_diag_cta_h(const MainParams p) {
         // staged: rows [0, row_in), column positions [0, col_in) relative to R0 / C0; a batch
         // at s0 needs columns < s0 + SB + NCC - 1 (pair slots and their high thresholds)
         int row_in = min(SB, nrows), col_in = min(SB, nrows) + NCC;
+        if (tma) tma_issue(R0, 0, row_in, C0, 0, col_in);
         stage(true, R0, 0, row_in);
         stage(false, C0, 0, col_in);
         cp_async_commit();
         cp_async_wait_all();
+        if (tma) { mbar_wait(bar, phase); phase ^= 1; }
         fixup(true, R0, 0, row_in);
         fixup(false, C0, 0, col_in);
         __syncthreads();
@@ -253,6 +310,7 @@ mp_diag_cta_h(const MainParams p) {
             }
             const int nxt = min(s0 + 2 * SB, nrows);
             const int r_lo = row_in, c_lo = col_in;
+            if (tma) tma_issue(R0, row_in, max(row_in, nxt), C0, col_in, max(col_in, nxt + NCC));
             stage(true, R0, row_in, nxt);
             stage(false, C0, col_in, nxt + NCC);
             row_in = max(row_in, nxt);
@@ -364,8 +422,10 @@ mp_diag_cta_h(const MainParams p) {
                 }
             }
             cp_async_wait_all();               // this thread's prefetch landed ...
+            if (tma) { mbar_wait(bar, phase); phase ^= 1; }   // ... and the batch's bulk copies
             fixup(true, R0, r_lo, row_in);     // ... so it converts the thresholds it staged
             fixup(false, C0, c_lo, col_in);
+            if (tma) fence_proxy_async();      // generic ring accesses before the next bulk copies
             __syncthreads();                   // publish; this batch's reads are all done
         }
     }

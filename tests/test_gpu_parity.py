@@ -385,7 +385,8 @@ def test_half_modes_ab_and_bands(ctx, oracle_mod, prec):
 
 @pytest.mark.parametrize("prec", ["fp16", "mixed", "fp16ck", "fp16c"])
 @pytest.mark.parametrize("shape", [(64, 2500, 32, 8, 61), (100, 400, 16, 4, 62), (200, 300, 16, 4, 63),
-                                   (64, 700, 32, -1, 64), (130, 300, 16, -1, 65)])
+                                   (64, 700, 32, -1, 64), (130, 300, 16, -1, 65), (71, 600, 24, 6, 66),
+                                   (71, 500, 16, -1, 67)])
 def test_half_modes_large_d(ctx, oracle_mod, prec, shape):
     """Large d in the half modes (block-cooperative half kernel, G = 8 / 16 / 32 lanes per
     pair): self-join (exclusion >= 0) and AB-join (-1), several tiles and ragged tails, vs the
