@@ -77,6 +77,7 @@ namespace mpk {
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int WARPS_PER_BLOCK = 4;
 constexpr unsigned DIRTY = 0x80000000u;
+constexpr unsigned EMPTY_IDX = 0x7FFFFFFFu;   // ring index of a slot without a local find
 
 // ------------------------------------------------------------------ precision traits
 template <class T> struct PT;
@@ -453,7 +454,7 @@ template <class T, int DL, int G, int W> struct Smem {
     using Gm = Geo<G, W>;
     static constexpr int D = DL * G;
     static constexpr size_t ring_bytes =
-        (((size_t)D * (Gm::PSR + Gm::PSC) * (sizeof(V4) + sizeof(typename KeyOps<T>::K))) + 15) & ~(size_t)15;
+        (((size_t)D * (Gm::PSR + Gm::PSC) * (sizeof(V4) + sizeof(unsigned))) + 15) & ~(size_t)15;
     static constexpr size_t flag_bytes = 0;  // dirty flags live in registers (bit masks)
     static constexpr size_t bytes_per_warp = ring_bytes + flag_bytes + (size_t)W * DL * 32 * sizeof(T);
     // warps per block: up to 4, fewer when a warp's rings are large (blocks <= ~112 KB)
@@ -492,8 +493,13 @@ mp_diag(const MainParams p) {
     V4* colv = rowv + (size_t)D * PSR;
     // ring keys: the warp's current (value, index) best of each staged (position, rank), the
     // index word's bit 31 marking it dirty; the .w words are filter hints only
-    K* rowi = reinterpret_cast<K*>(colv + (size_t)D * PSC);
-    K* coli = rowi + (size_t)D * PSR;
+    // ring indices: the index of the warp's own best (value in the slot's .w) of a staged
+    // (position, rank), DIRTY when it improved on the staged global key; EMPTY_IDX until then.
+    // Only locally found indices live here -- the global key's index is never staged, so a key
+    // updated by another warp between its value and index reads cannot pair a value with a
+    // foreign index (a tie with the staged value is taken locally and settled by the merge).
+    unsigned* rowi = reinterpret_cast<unsigned*>(colv + (size_t)D * PSC);
+    unsigned* coli = rowi + (size_t)D * PSR;
     // dirty ring slots: warp-uniform bit masks in registers (slot -> bit), set after each
     // slow path by a warp OR-reduction, cleared on eviction -- no shared-memory flags to poll
     static_assert(Gm::RING_R <= 64 && Gm::RING_C <= 64, "dirty masks hold one bit per ring slot");
@@ -533,7 +539,7 @@ mp_diag(const MainParams p) {
         const int cnt = p_hi - p_lo;
         if (cnt <= 0) return;
         V4* buf = is_row ? rowv : colv;
-        K* ib = is_row ? rowi : coli;
+        unsigned* ib = is_row ? rowi : coli;
         const int ps = is_row ? PSR : PSC;
         const V4* __restrict__ st = is_row ? st_q : st_r;
         const bool want_thr = is_row || SELF;
@@ -552,7 +558,8 @@ mp_diag(const MainParams p) {
                     cp_async16(dst, src);
                     cp_async8(&dst->z, &src->z);
                 }
-                KO::stage(keys + (size_t)pos * d + rank_of_plane<DL, G>(pl), &dst->w, &ib[pl * ps + sl]);
+                cp_async4(&dst->w, reinterpret_cast<const char*>(keys + (size_t)pos * d + rank_of_plane<DL, G>(pl)) + 4);
+                ib[pl * ps + sl] = EMPTY_IDX;
             }
             return;
         }
@@ -576,10 +583,11 @@ mp_diag(const MainParams p) {
             }
             const int rk = rank_of_plane<DL, G>(pl);
             if (rk < d && want_thr) {
-                KO::stage(keys + (size_t)pos * d + rk, &dst->w, &ib[pl * ps + sl]);
+                cp_async4(&dst->w, reinterpret_cast<const char*>(keys + (size_t)pos * d + rk) + 4);
+                ib[pl * ps + sl] = EMPTY_IDX;
             } else {
                 dst->w = NINF;  // never hit
-                ib[pl * ps + sl] = EMPTY32;
+                ib[pl * ps + sl] = EMPTY_IDX;
             }
         }
     };
@@ -588,7 +596,7 @@ mp_diag(const MainParams p) {
         const int cnt = p_hi - p_lo;
         if (cnt <= 0) return;
         const V4* buf = is_row ? rowv : colv;
-        const K* ib = is_row ? rowi : coli;
+        const unsigned* ib = is_row ? rowi : coli;
         const int ps = is_row ? PSR : PSC;
         // early out (warp-uniform, registers only): most evictions find nothing dirty
         DMask& dm = is_row ? dmask_r : dmask_c;
@@ -609,8 +617,9 @@ mp_diag(const MainParams p) {
             if (((dirty >> sl) & 1ull) == 0) continue;
             const int rk = rank_of_plane<DL, G>(pl);
             if (rk >= d) continue;
-            const K kv = ib[pl * ps + sl];
-            if (kv & DIRTY) atomicMin(keys + (size_t)pos * d + rk, kv & ~(K)DIRTY);
+            const unsigned kv = ib[pl * ps + sl];
+            if (kv & DIRTY)   // the slot's .w is the value of the warp's best (set with the index)
+                atomicMin(keys + (size_t)pos * d + rk, ((K)__float_as_uint(buf[pl * ps + sl].w) << 32) | (kv & ~DIRTY));
         }
     };
 
@@ -857,12 +866,11 @@ mp_diag(const MainParams p) {
                         for (int u = W - 1; u >= 0; --u)
                             if (v[u] == vr) j = col[u];                 // lowest column first
                         const int ix = pl * PSR + sr;
-                        const K kc = rowi[ix];
-                        const T cur = __uint_as_float((unsigned)(kc >> 32));
-                        const unsigned ci = (unsigned)kc & ~DIRTY;
+                        const T cur = rowv[ix].w;
+                        const unsigned ci = rowi[ix] & ~DIRTY;
                         if (vr < cur || (vr == cur && (unsigned)j < ci)) {
                             rowv[ix].w = vr;
-                            rowi[ix] = ((K)__float_as_uint(vr) << 32) | (unsigned)j | DIRTY;
+                            rowi[ix] = (unsigned)j | DIRTY;
                             mark_r |= 1ull << sr;
                         }
                     }
@@ -878,12 +886,11 @@ mp_diag(const MainParams p) {
                             if (vc < INF && eqc != 0 && lane == 31 - __clz(eqc)) {
                                 const int scu = Gm::scol(col[u]);
                                 const int ix = pl * PSC + scu;
-                                const K kc = coli[ix];
-                                const T cur = __uint_as_float((unsigned)(kc >> 32));
-                                const unsigned ci = (unsigned)kc & ~DIRTY;
+                                const T cur = colv[ix].w;
+                                const unsigned ci = coli[ix] & ~DIRTY;
                                 if (vc < cur || (vc == cur && (unsigned)row < ci)) {
                                     colv[ix].w = vc;
-                                    coli[ix] = ((K)__float_as_uint(vc) << 32) | (unsigned)row | DIRTY;
+                                    coli[ix] = (unsigned)row | DIRTY;
                                     mark_c |= 1ull << scu;
                                 }
                             }
