@@ -603,7 +603,7 @@ struct Side {
 
 struct Streamer {
     // MP_STREAM_PROFILE=1: host seconds per phase, printed to stderr at the end of the call
-    double t_sync = 0, t_remap = 0, t_pre = 0, t_fin = 0;
+    double t_sync = 0, t_remap = 0, t_pre = 0, t_fin = 0, t_save = 0, t_unmap = 0, t_map = 0;
     static double now() {
         return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
     }
@@ -649,11 +649,16 @@ struct Streamer {
                 gi = ge;
             }
             if (any) MP_CUDA(ctx, cudaStreamSynchronize(s));
+            t_save += now() - t0;
         }
+        const double tu = now();
         static const char* keep_env = std::getenv("MP_STREAM_NOUNMAP");   // debugging knob: "1" or an array name
         const bool keep_all = keep_env && (std::strcmp(keep_env, "1") == 0 || std::strcmp(keep_env, a.name) == 0);
         for (size_t gi = 0; gi < ng && !keep_all; ++gi)
             if (a.h[gi] && !nm[gi]) MP_CU(ctx, vm.unmap_g(a, gi));
+        const double tm = now();
+        t_unmap += tm - tu;
+        struct AccM { double& t; double t0; ~AccM() { t += now() - t0; } } accm{t_map, tm};
         for (size_t gi = 0; gi < ng;) {   // map the new granules, one access call and copy per run
             if (a.h[gi] || !nm[gi]) { ++gi; continue; }
             size_t ge = gi;
@@ -965,8 +970,8 @@ mp_status run_stream(mp_ctx* ctx, const double* T, const double* Tr, int64_t d, 
         ++ei;
     }
     if (std::getenv("MP_STREAM_PROFILE"))
-        std::fprintf(stderr, "mp_compute_stream: host s sync %.3f remap %.3f precompute %.3f finalize %.3f\n", S.t_sync,
-                     S.t_remap, S.t_pre, S.t_fin);
+        std::fprintf(stderr, "mp_compute_stream: host s sync %.3f remap %.3f (key saves %.3f unmap %.3f map+restore %.3f) "
+                     "precompute %.3f finalize %.3f\n", S.t_sync, S.t_remap, S.t_save, S.t_unmap, S.t_map, S.t_pre, S.t_fin);
     MP_CUDA(ctx, cudaStreamSynchronize(s));
     double tot = 0;
     for (size_t k = 0; k + 1 < evs.size(); k += 2) {
