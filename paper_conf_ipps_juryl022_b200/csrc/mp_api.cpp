@@ -498,6 +498,23 @@ struct Vmm {
         return CUDA_SUCCESS;
     }
     CUresult set_access(VArr& a, size_t g0, size_t g1) { return access(a.base + g0 * gran, (g1 - g0) * gran, &acc, 1); }
+    // unmap granules [g0, g1) (each mapped separately) with one call; per granule if the driver
+    // refuses a range spanning several mappings
+    CUresult unmap_run(VArr& a, size_t g0, size_t g1) {
+        if (g1 - g0 > 1 && multi_unmap) {
+            if (unmap(a.base + g0 * gran, (g1 - g0) * gran) == CUDA_SUCCESS) {
+                for (size_t g = g0; g < g1; ++g) { pool.push_back(a.h[g]); a.h[g] = 0; mapped -= gran; }
+                return CUDA_SUCCESS;
+            }
+            multi_unmap = false;
+        }
+        for (size_t g = g0; g < g1; ++g) {
+            CUresult r = unmap_g(a, g);
+            if (r != CUDA_SUCCESS) return r;
+        }
+        return CUDA_SUCCESS;
+    }
+    bool multi_unmap = true;
     CUresult unmap_g(VArr& a, size_t g) {
         CUresult r = unmap(a.base + g * gran, gran);
         pool.push_back(a.h[g]);
@@ -654,8 +671,13 @@ struct Streamer {
         const double tu = now();
         static const char* keep_env = std::getenv("MP_STREAM_NOUNMAP");   // debugging knob: "1" or an array name
         const bool keep_all = keep_env && (std::strcmp(keep_env, "1") == 0 || std::strcmp(keep_env, a.name) == 0);
-        for (size_t gi = 0; gi < ng && !keep_all; ++gi)
-            if (a.h[gi] && !nm[gi]) MP_CU(ctx, vm.unmap_g(a, gi));
+        for (size_t gi = 0; gi < ng && !keep_all;) {   // unmap the leaving granules, one call per run
+            if (!(a.h[gi] && !nm[gi])) { ++gi; continue; }
+            size_t ge = gi;
+            while (ge < ng && a.h[ge] && !nm[ge]) ++ge;
+            MP_CU(ctx, vm.unmap_run(a, gi, ge));
+            gi = ge;
+        }
         const double tm = now();
         t_unmap += tm - tu;
         struct AccM { double& t; double t0; ~AccM() { t += now() - t0; } } accm{t_map, tm};
