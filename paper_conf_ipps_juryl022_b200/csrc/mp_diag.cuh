@@ -328,12 +328,6 @@ constexpr long long EXT_EMPTY = 0x7FFFFFFFFFFFFFFFll;                  // INT64_
 template <class T> struct KeyOps;
 template <> struct KeyOps<float> {
     using K = unsigned long long;
-    // async-stage the key's value (high word) into the threshold hint thr and the whole key
-    // (one 8-byte copy: value and index always from the same atomicMin state) into key
-    static __device__ __forceinline__ void stage(const K* p, float* thr, K* key) {
-        cp_async4(thr, reinterpret_cast<const char*>(p) + 4);
-        cp_async8(key, p);
-    }
     static __device__ __forceinline__ void merge(K* p, float v, unsigned i) {
         atomicMin(p, ((K)__float_as_uint(v) << 32) | (K)i);
     }
