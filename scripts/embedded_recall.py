@@ -7,7 +7,7 @@ occurrence start x and every dimension count k, the matrix-profile index I[k][x]
 ANOTHER occurrence of the pattern:
   R_embedded      strict: I[k][x] is another occurrence's start,
   R^r_embedded    relaxed with factor r: within r*m of another occurrence's start (L917-931).
-Modes: FP64 (the reference), FP32, Mixed, FP16C, FP16.  Writes profiles/r2_embedded_recall.json.
+Modes: FP64 (the reference), FP32, Mixed, FP16CK, FP16C, FP16.  Writes profiles/r2_embedded_recall.json.
     python scripts/embedded_recall.py
 """
 import json
